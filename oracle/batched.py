@@ -1,0 +1,83 @@
+"""fp64 *batched* executor: runs an explicit schedule of batched tasks, each task executing
+its rows as one stacked matrix contraction, exactly as cellular batching does (§3.1:
+cells of the same type with no data dependency between them are batched together).
+
+TEST INFRASTRUCTURE ONLY. Used by tests/test_oracle_batching.py (pin P4) to check by brute
+force that every dependency-respecting batching schedule reaches the unbatched result of
+oracle.cells (the method is exact: batching only concatenates independent rows).
+"""
+from __future__ import annotations
+
+from typing import Dict, List, Sequence, Tuple
+
+import numpy as np
+
+from .cells import f64, sigmoid
+
+
+def _lstm_rows(W, b, X, Hp, Cp):
+    H = Hp.shape[1]
+    Z = np.concatenate([X, Hp], axis=1) @ f64(W).T + f64(b)
+    i, f = sigmoid(Z[:, :H]), sigmoid(Z[:, H:2 * H])
+    g, o = np.tanh(Z[:, 2 * H:3 * H]), sigmoid(Z[:, 3 * H:])
+    C = f * Cp + i * g
+    return o * np.tanh(C), C
+
+
+def run_chain_schedule(w, token_lists: Sequence[Sequence[int]],
+                       schedule: Sequence[Sequence[Tuple[int, int]]]):
+    """schedule: list of tasks, each a list of (request, step) rows. Single-layer or stacked
+    LSTM: each row runs one full timestep of the stack. Returns {request: (h list, c list)}."""
+    Hd, L = w.hidden, w.layers
+    h = {r: [np.zeros(Hd) for _ in range(L)] for r in range(len(token_lists))}
+    c = {r: [np.zeros(Hd) for _ in range(L)] for r in range(len(token_lists))}
+    done = {r: 0 for r in range(len(token_lists))}
+    for task in schedule:
+        rows = list(task)
+        for r, k in rows:
+            assert done[r] == k, "schedule violates chain order"
+        X = np.stack([f64(w.E[int(token_lists[r][k])]) for r, k in rows])
+        for l in range(L):
+            Hp = np.stack([h[r][l] for r, _ in rows])
+            Cp = np.stack([c[r][l] for r, _ in rows])
+            Hn, Cn = _lstm_rows(w.W[l], w.b[l], X, Hp, Cp)
+            for j, (r, _) in enumerate(rows):
+                h[r][l], c[r][l] = Hn[j], Cn[j]
+            X = Hn
+        for r, _ in rows:
+            done[r] += 1
+    return {r: (h[r], c[r]) for r in h}
+
+
+def run_tree_schedule(w, trees: Sequence[Tuple[Sequence[int], Sequence[int], Sequence[int]]],
+                      schedule: Sequence[Sequence[Tuple[int, int]]]):
+    """trees: list of (tokens, left, right) in post-order. schedule: tasks of (tree, node)
+    rows; a task holds only leaves or only internal nodes (two cell types, L99, L383).
+    Returns {tree: (root_h, root_c)}."""
+    Hd = w.hidden
+    st: Dict[Tuple[int, int], Tuple[np.ndarray, np.ndarray]] = {}
+    for task in schedule:
+        rows = list(task)
+        leaf = [trees[t][1][v] < 0 for t, v in rows]
+        assert all(leaf) or not any(leaf), "mixed cell types in one task"
+        if all(leaf):
+            X = np.stack([f64(w.E[int(trees[t][0][v])]) for t, v in rows])
+            Z = X @ f64(w.W_leaf).T + f64(w.b_leaf)
+            i, o, u = sigmoid(Z[:, :Hd]), sigmoid(Z[:, Hd:2 * Hd]), np.tanh(Z[:, 2 * Hd:])
+            C = i * u
+            Hn = o * np.tanh(C)
+        else:
+            for t, v in rows:
+                assert (t, trees[t][1][v]) in st and (t, trees[t][2][v]) in st, "dependency"
+            HL = np.stack([st[(t, trees[t][1][v])][0] for t, v in rows])
+            CL = np.stack([st[(t, trees[t][1][v])][1] for t, v in rows])
+            HR = np.stack([st[(t, trees[t][2][v])][0] for t, v in rows])
+            CR = np.stack([st[(t, trees[t][2][v])][1] for t, v in rows])
+            Z = np.concatenate([HL, HR], axis=1) @ f64(w.U).T + f64(w.b_int)
+            i, fL, fR = sigmoid(Z[:, :Hd]), sigmoid(Z[:, Hd:2 * Hd]), sigmoid(Z[:, 2 * Hd:3 * Hd])
+            o, u = sigmoid(Z[:, 3 * Hd:4 * Hd]), np.tanh(Z[:, 4 * Hd:])
+            C = i * u + fL * CL + fR * CR
+            Hn = o * np.tanh(C)
+        for j, (t, v) in enumerate(rows):
+            st[(t, v)] = (Hn[j], C[j])
+    return {t: st[(t, len(trees[t][1]) - 1)] for t in range(len(trees))}

@@ -1,0 +1,411 @@
+"""Replay oracle for BatchMaker's scheduler: Algorithm 1 + request processor + slot pool,
+driven in virtual time.
+
+TEST INFRASTRUCTURE ONLY (see oracle/__init__.py). Independent of the C++ engine: the two
+share no code; tests compare the engine's task log with this replay bit for bit (P9).
+
+Algorithm 1 is followed line by line in `Schedule`, `Batch` and
+`FormBatchedTask`; the surrounding prose it depends on:
+  * request processor unfolds a request into a cell graph and subgraphs ........ L323, L341
+  * Seq2Seq = encoder subgraph + decoder subgraph; TreeLSTM = one subgraph per leaf
+    + one subgraph for all internal nodes, passed on when all leaves finish ...... L341, L383-L385
+  * Schedule runs whenever a worker becomes idle ................................ L371
+  * node dependencies are updated at submission (L381: UpdateNodesDependency);
+    inter-subgraph dependencies are released at completion ..................... L331, L385
+  * pin a subgraph to the worker; unpin when its in-flight task counter is 0 ..... L381
+  * MaxTasksToSubmit default 5 .................................................. L379
+Readings where the paper is silent (listed in DESIGN.md):
+  S13 line 5 uses ">= Bsizes.Max()" (pseudo-code wins over prose)
+  S14 Bsizes.Max() = the cell type's bmax; Bsizes.Min() = min_followon
+  S15 an empty batch ends Batch (never submitted)
+  S16 NumReadyNodes counts every ready node of the cell type
+  S17 NumRunningTasks = tasks of the type submitted and not yet retired
+  S18 subgraph queue FIFO by enqueue event (ties: request id, subgraph id); ready nodes
+      within a subgraph in ascending (height, post-order index)
+  S19 "idle" = outstanding tasks <= k (k = 0 is the paper's idle)
+  S20 intra-subgraph successors ready at submit; inter-subgraph at retire
+  S21 same-tick order: retire (FIFO) -> admit arrivals (trace order) -> Schedule if idle;
+      every task takes one tick on the single worker
+  S22 slots: lowest free index. A request takes all the slots it will ever need when its
+      first node is scheduled: chain/seq2seq one slot (all layers, encoder and decoder
+      share it), trees one slot per node (assigned in post-order index order). All are
+      freed at request completion. Taking them up front makes the pool deadlock-free (a
+      started request can always finish). A request whose slots are not available is
+      skipped (its subgraph stays queued); if that leaves the chosen cell type with an
+      empty batch, Schedule moves on to its next choice.
+"""
+from __future__ import annotations
+
+import bisect
+import dataclasses
+from collections import deque
+from typing import Dict, List, Optional, Sequence, Tuple
+
+CHAIN, SEQ2SEQ, TREE = 0, 1, 2
+
+
+@dataclasses.dataclass
+class CellType:
+    id: int
+    bmax: int
+    priority: int
+    queue: List["Subgraph"] = dataclasses.field(default_factory=list)
+    running_tasks: int = 0
+
+    def num_ready_nodes(self) -> int:
+        return sum(len(sg.ready) for sg in self.queue)
+
+
+class Subgraph:
+    def __init__(self, req: "Req", sid: int, ct: CellType, nodes: List[int]):
+        self.req, self.sid, self.ct = req, sid, ct
+        self.nodes = nodes                 # node ids (request-local) of this subgraph
+        self.ready: List[int] = []         # ready, not yet submitted, sorted by key
+        self.n_submitted = 0
+        self.n_completed = 0
+        self.pinned: Optional[int] = None
+        self.inflight = 0                  # tasks in flight holding nodes of this subgraph
+
+
+class Req:
+    def __init__(self, rid: int, kind: int, n_nodes: int):
+        self.rid, self.kind = rid, kind
+        self.n_nodes = n_nodes
+        self.n_completed = 0
+        self.slots: Dict[int, int] = {}    # node -> slot (trees) ; -1 -> slot (chain/s2s)
+        self.subgraphs: List[Subgraph] = []
+        self.complete_tick: Optional[float] = None
+        self.first_tick: Optional[float] = None
+        # structure
+        self.left: Optional[Sequence[int]] = None
+        self.right: Optional[Sequence[int]] = None
+        self.parent: List[int] = []
+        self.height: List[int] = []
+        self.submitted: List[bool] = [False] * n_nodes
+        self.node_sg: List[Subgraph] = [None] * n_nodes  # type: ignore
+        self.leaves_left = 0
+        self.enc_len = 0
+        self.internal_sg: Optional[Subgraph] = None
+
+
+class SlotPool:
+    """Lowest-free-index allocator (reading S22)."""
+
+    def __init__(self, n: int):
+        self.free = list(range(n))   # sorted
+
+    def available(self) -> int:
+        return len(self.free)
+
+    def alloc(self) -> int:
+        return self.free.pop(0)
+
+    def release(self, s: int):
+        bisect.insort(self.free, s)
+
+
+@dataclasses.dataclass
+class TaskRow:
+    rid: int
+    node: int
+    slot: int
+
+
+@dataclasses.dataclass
+class Task:
+    index: int
+    ct: int
+    worker: int
+    tick: float                    # submission tick
+    rows: List[TaskRow]
+    finish: float = 0.0
+
+
+class Replay:
+    """Algorithm 1 with one worker per engine (S23), driven by `run()` in virtual time."""
+
+    def __init__(self, cell_types: Sequence[Tuple[int, int]], max_slots: int = 1 << 20,
+                 max_tasks_to_submit: int = 5, min_followon: int = 1,
+                 schedule_when_outstanding_leq: int = 0):
+        # cell_types: list of (bmax, priority); cell id = position
+        self.cts = [CellType(i, bm, pr) for i, (bm, pr) in enumerate(cell_types)]
+        self.pool = SlotPool(max_slots)
+        self.max_tasks = max_tasks_to_submit
+        self.min_followon = min_followon
+        self.k = schedule_when_outstanding_leq
+        self.reqs: List[Req] = []
+        self.tasks: List[Task] = []
+        self.inflight: deque = deque()
+        self.completions: List[Tuple[int, float]] = []   # (rid, tick) in completion order
+        self.now = 0.0
+        self.last_finish = 0.0
+
+    # ------------------------------------------------------------ request processor (A1)
+    def admit(self, kind: int, cells: Sequence[int], length: int = 0, decode_len: int = 0,
+              left: Optional[Sequence[int]] = None, right: Optional[Sequence[int]] = None) -> int:
+        rid = len(self.reqs)
+        if kind == CHAIN:
+            r = Req(rid, kind, length)
+            sg = Subgraph(r, 0, self.cts[cells[0]], list(range(length)))
+            r.subgraphs = [sg]
+            for v in range(length):
+                r.node_sg[v] = sg
+            r.height = list(range(length))
+            self._enqueue(sg)
+            sg.ready = [0]
+        elif kind == SEQ2SEQ:
+            r = Req(rid, kind, length + decode_len)
+            r.enc_len = length
+            enc = Subgraph(r, 0, self.cts[cells[0]], list(range(length)))
+            dec = Subgraph(r, 1, self.cts[cells[1]], list(range(length, length + decode_len)))
+            r.subgraphs = [enc, dec]
+            for v in range(length):
+                r.node_sg[v] = enc
+            for v in range(length, length + decode_len):
+                r.node_sg[v] = dec
+            r.height = list(range(length + decode_len))
+            self._enqueue(enc)
+            enc.ready = [0]
+        elif kind == TREE:
+            n = len(left)
+            r = Req(rid, kind, n)
+            r.left, r.right = list(left), list(right)
+            r.parent = [-1] * n
+            r.height = [0] * n
+            for v in range(n):
+                if left[v] >= 0:
+                    r.parent[left[v]] = v
+                    r.parent[right[v]] = v
+                    r.height[v] = 1 + max(r.height[left[v]], r.height[right[v]])
+            leaves = [v for v in range(n) if left[v] < 0]
+            internal = [v for v in range(n) if left[v] >= 0]
+            r.leaves_left = len(leaves)
+            sid = 0
+            for v in leaves:
+                sg = Subgraph(r, sid, self.cts[cells[0]], [v])
+                sid += 1
+                r.node_sg[v] = sg
+                r.subgraphs.append(sg)
+            if internal:
+                isg = Subgraph(r, sid, self.cts[cells[1]], internal)
+                for v in internal:
+                    r.node_sg[v] = isg
+                r.subgraphs.append(isg)
+                r.internal_sg = isg
+            for sg in r.subgraphs[:len(leaves)]:
+                self._enqueue(sg)
+                sg.ready = [sg.nodes[0]]
+        else:
+            raise ValueError(kind)
+        self.reqs.append(r)
+        return rid
+
+    def _enqueue(self, sg: Subgraph):
+        sg.ct.queue.append(sg)
+
+    def _node_key(self, r: Req, v: int):
+        return (r.height[v], v)
+
+    # ------------------------------------------------------------ Algorithm 1
+    def schedule(self, worker: int = 0) -> List[Task]:
+        """Schedule(worker), Algorithm 1 lines 4-11. Reading S22: if the chosen type forms
+        no task only because the slot pool is exhausted, Schedule falls through to the next
+        choice among the remaining types (the paper has no slot pool)."""
+        cand = list(self.cts)
+        while cand:
+            S = [ct for ct in cand if ct.num_ready_nodes() >= ct.bmax]         # line 5 (S13)
+            if not S:
+                S = [ct for ct in cand
+                     if ct.running_tasks == 0 and ct.num_ready_nodes() > 0]  # line 7
+            if not S:
+                S = [ct for ct in cand if ct.num_ready_nodes() > 0]          # line 9
+            if not S:
+                return []
+            ct = max(S, key=lambda c: (c.priority, -c.id))                    # line 10
+            tasks = self.batch(ct, worker)                                    # line 11
+            if tasks:
+                return tasks
+            cand.remove(ct)
+        return []
+
+    def batch(self, ct: CellType, worker: int) -> List[Task]:
+        """Batch(ct, worker), Algorithm 1 lines 12-23."""
+        out = []
+        num_tasks = 0                                                          # line 13
+        while num_tasks < self.max_tasks:                                      # line 14
+            batch = self.form_batched_task(ct, worker)                         # line 15
+            if not batch:                                                      # S15
+                break
+            if len(batch) >= self.min_followon or num_tasks == 0:              # line 16
+                out.append(self.submit(ct, batch, worker))                     # lines 17-18
+                num_tasks += 1                                                 # line 19
+                # lines 20-21: pinning happens inside submit()
+            else:
+                break                                                          # line 23
+        return out
+
+    def form_batched_task(self, ct: CellType, worker: int) -> List[Tuple[Subgraph, int]]:
+        """FormBatchedTask(ct, worker), Algorithm 1 lines 24-32, plus the slot check (S22).
+        Pure: nothing is consumed until submit()."""
+        batch: List[Tuple[Subgraph, int]] = []                                 # line 25
+        free = self.pool.available()
+        for sg in ct.queue:                                                    # line 26
+            if sg.pinned is not None and sg.pinned != worker:                  # line 27
+                continue
+            for v in sg.ready:                                                 # line 28
+                # a request not started yet needs all its slots (S22): n for trees, else 1
+                r = sg.req
+                need = 0
+                if not r.slots and not any(s.req is r for s, _ in batch):
+                    need = r.n_nodes if r.kind == TREE else 1
+                if need > free:
+                    break                                                      # S22 skip
+                free -= need
+                batch.append((sg, v))                                          # line 29
+                if len(batch) == ct.bmax:                                      # line 30
+                    return batch                                               # line 31
+        return batch                                                           # line 32
+
+    def submit(self, ct: CellType, batch, worker: int) -> Task:
+        rows = []
+        touched = []
+        for sg, v in batch:
+            r = sg.req
+            if not r.slots:
+                if r.kind == TREE:
+                    for u in range(r.n_nodes):
+                        r.slots[u] = self.pool.alloc()
+                else:
+                    r.slots[-1] = self.pool.alloc()
+            slot = r.slots[v] if r.kind == TREE else r.slots[-1]
+            if r.first_tick is None:
+                r.first_tick = self.now
+            rows.append(TaskRow(r.rid, v, slot))
+            sg.ready.remove(v)
+            sg.n_submitted += 1
+            r.submitted[v] = True
+            if sg not in touched:
+                touched.append(sg)
+        task = Task(len(self.tasks), ct.id, worker, self.now, rows)
+        self.tasks.append(task)
+        ct.running_tasks += 1
+        # UpdateNodesDependency (line 18): intra-subgraph successors become ready now (S20)
+        for sg, v in batch:
+            self._release_successor(sg, v)
+        for sg in touched:
+            sg.inflight += 1
+            sg.pinned = worker                                                 # line 21
+            if sg.n_submitted == len(sg.nodes):
+                ct.queue.remove(sg)
+        return task
+
+    def _release_successor(self, sg: Subgraph, v: int):
+        r = sg.req
+        if r.kind in (CHAIN, SEQ2SEQ):
+            nxt = v + 1
+            if nxt < r.n_nodes and r.node_sg[nxt] is sg:
+                self._make_ready(sg, nxt)
+        else:
+            p = r.parent[v]
+            if p >= 0 and r.node_sg[p] is sg and not r.submitted[p] and p not in sg.ready:
+                if r.submitted[r.left[p]] and r.submitted[r.right[p]]:
+                    self._make_ready(sg, p)
+
+    def _make_ready(self, sg: Subgraph, v: int):
+        keys = [self._node_key(sg.req, u) for u in sg.ready]
+        i = bisect.bisect(keys, self._node_key(sg.req, v))
+        sg.ready.insert(i, v)
+
+    # ------------------------------------------------------------ completion (A13)
+    def retire(self, task: Task):
+        ct = self.cts[task.ct]
+        ct.running_tasks -= 1
+        seen = []
+        for row in task.rows:
+            r = self.reqs[row.rid]
+            sg = r.node_sg[row.node]
+            if sg not in seen:
+                seen.append(sg)
+                sg.inflight -= 1
+                if sg.inflight == 0:
+                    sg.pinned = None
+            sg.n_completed += 1
+            r.n_completed += 1
+            if sg.n_completed == len(sg.nodes):
+                self._subgraph_done(sg)
+            if r.n_completed == r.n_nodes:
+                r.complete_tick = self.now
+                self.completions.append((r.rid, self.now))
+                for s in sorted(set(r.slots.values())):
+                    self.pool.release(s)
+
+    def _subgraph_done(self, sg: Subgraph):
+        r = sg.req
+        if r.kind == SEQ2SEQ and sg.sid == 0 and len(r.subgraphs[1].nodes) > 0:
+            dec = r.subgraphs[1]
+            self._enqueue(dec)
+            dec.ready = [dec.nodes[0]]
+        elif r.kind == TREE and r.left[sg.nodes[0]] < 0:
+            r.leaves_left -= 1
+            if r.leaves_left == 0 and r.internal_sg is not None:
+                isg = r.internal_sg
+                self._enqueue(isg)
+                for v in isg.nodes:
+                    if r.submitted[r.left[v]] and r.submitted[r.right[v]]:
+                        self._make_ready(isg, v)
+
+    # ------------------------------------------------------------ virtual-time driver (S21)
+    def run(self, requests: Sequence[dict], max_ticks: float = 1e9):
+        """requests: dicts with keys kind, cells, arrival, length / decode_len / left, right.
+        Admission order = list order. Returns self (tasks, completions filled)."""
+        pending = list(range(len(requests)))
+        rid_of = {}
+        t = 0.0
+        while True:
+            self.now = t
+            while self.inflight and self.inflight[0].finish <= t:
+                self.retire(self.inflight.popleft())
+            still = []
+            for i in pending:
+                q = requests[i]
+                if q["arrival"] <= t:
+                    rid_of[i] = self.admit(q["kind"], q["cells"], q.get("length", 0),
+                                           q.get("decode_len", 0), q.get("left"), q.get("right"))
+                else:
+                    still.append(i)
+            pending = still
+            if len(self.inflight) <= self.k:
+                for task in self.schedule(0):
+                    start = max(t, self.last_finish)
+                    task.finish = start + 1
+                    self.last_finish = task.finish
+                    self.inflight.append(task)
+            cand = []
+            if self.inflight:
+                cand.append(self.inflight[0].finish)
+            if pending:
+                cand.append(min(requests[i]["arrival"] for i in pending))
+            if not cand:
+                break
+            nt = min(cand)
+            assert nt > t
+            t = nt
+            if t > max_ticks:
+                raise RuntimeError("replay did not terminate")
+        return self
+
+
+def replay_requests(reqs, cells_for_kind, **kw) -> Replay:
+    """Convenience: build the request dicts from workloads.gen.Request objects."""
+    cts = kw.pop("cell_types")
+    rp = Replay(cts, **kw)
+    qs = []
+    for q in reqs:
+        d = {"kind": q.kind, "cells": cells_for_kind[q.kind], "arrival": q.arrival}
+        if q.kind == TREE:
+            d["left"], d["right"] = q.left, q.right
+        else:
+            d["length"] = q.length
+            d["decode_len"] = q.decode_len
+        qs.append(d)
+    return rp.run(qs)
