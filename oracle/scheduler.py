@@ -24,8 +24,10 @@ Readings where the paper is silent (listed in DESIGN.md):
       within a subgraph in ascending (height, post-order index)
   S19 "idle" = outstanding tasks <= k (k = 0 is the paper's idle)
   S20 intra-subgraph successors ready at submit; inter-subgraph at retire
-  S21 same-tick order: retire (FIFO) -> admit arrivals (trace order) -> Schedule if idle;
-      every task takes one tick on the single worker
+  S21 same-tick order: retire (FIFO) -> admit arrivals -> Schedule if idle; every task
+      takes one tick on the single worker. Admission is FIFO in submission order: a request
+      is admitted once its arrival time has passed and every earlier-submitted request has
+      been admitted (identical to "all due arrivals in trace order" for sorted traces).
   S22 slots: lowest free index. A request takes all the slots it will ever need when its
       first node is scheduled: chain/seq2seq one slot (all layers, encoder and decoder
       share it), trees one slot per node (assigned in post-order index order). All are
@@ -365,15 +367,11 @@ class Replay:
             self.now = t
             while self.inflight and self.inflight[0].finish <= t:
                 self.retire(self.inflight.popleft())
-            still = []
-            for i in pending:
+            while pending and requests[pending[0]]["arrival"] <= t:
+                i = pending.pop(0)
                 q = requests[i]
-                if q["arrival"] <= t:
-                    rid_of[i] = self.admit(q["kind"], q["cells"], q.get("length", 0),
-                                           q.get("decode_len", 0), q.get("left"), q.get("right"))
-                else:
-                    still.append(i)
-            pending = still
+                rid_of[i] = self.admit(q["kind"], q["cells"], q.get("length", 0),
+                                       q.get("decode_len", 0), q.get("left"), q.get("right"))
             if len(self.inflight) <= self.k:
                 for task in self.schedule(0):
                     start = max(t, self.last_finish)
@@ -384,7 +382,7 @@ class Replay:
             if self.inflight:
                 cand.append(self.inflight[0].finish)
             if pending:
-                cand.append(min(requests[i]["arrival"] for i in pending))
+                cand.append(requests[pending[0]]["arrival"])
             if not cand:
                 break
             nt = min(cand)

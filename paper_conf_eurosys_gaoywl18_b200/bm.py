@@ -1,0 +1,312 @@
+"""Thin ctypes binding of the C-ABI in include/bm.h (libbm.so): argument marshalling only.
+
+Every step of the hot path runs inside libbm.so (C++ scheduler + sm_100a kernels). There is
+no Python or CPU fallback: if libbm.so is missing this module raises at import, and on a
+machine without an sm_100 GPU bm_create fails with BM_E_NODEV (except the BM_CLOCK_DRY
+scheduler-only mode, which never touches a device).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from typing import List, Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbm.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with "
+                      "`python -m paper_conf_eurosys_gaoywl18_b200.build` (no CPU fallback exists)")
+lib = C.CDLL(LIB_PATH)
+
+# ---------------------------------------------------------------- constants (bm.h)
+OK, E_INVAL, E_NOMEM, E_FULL, E_AGAIN, E_CUDA, E_STATE, E_NODEV = 0, -1, -2, -3, -4, -5, -6, -7
+PREC_BF16, PREC_FP32 = 0, 1
+CLOCK_WALL, CLOCK_VIRTUAL, CLOCK_DRY = 0, 1, 2
+CELL_LSTM, CELL_LSTM_PROJ, CELL_TREE_LEAF, CELL_TREE_INTERNAL = 0, 1, 2, 3
+REQ_CHAIN, REQ_SEQ2SEQ, REQ_TREE = 0, 1, 2
+ROW_FIRST, ROW_LAST, ROW_PARITY = 1, 2, 4
+
+
+class Config(C.Structure):
+    _fields_ = [(n, C.c_int) for n in (
+        "device", "precision", "clock", "hidden", "pool_layers", "max_slots", "max_requests",
+        "max_tasks_to_submit", "min_followon_batch", "schedule_when_outstanding_leq",
+        "max_decode_len", "keep_results", "record_logits", "time_kernels")]
+
+
+class CellDesc(C.Structure):
+    _fields_ = [(n, C.c_int) for n in ("kind", "hidden", "layers", "vocab", "max_batch", "priority")]
+
+
+class Weights(C.Structure):
+    _fields_ = [("W", C.POINTER(C.POINTER(C.c_float))), ("b", C.POINTER(C.POINTER(C.c_float))),
+                ("E", C.POINTER(C.c_float)), ("W_out", C.POINTER(C.c_float)),
+                ("b_out", C.POINTER(C.c_float))]
+
+
+class Request(C.Structure):
+    _fields_ = [("kind", C.c_int), ("cell0", C.c_int), ("cell1", C.c_int), ("n", C.c_int),
+                ("tokens", C.POINTER(C.c_int32)), ("decode_len", C.c_int),
+                ("left", C.POINTER(C.c_int32)), ("right", C.POINTER(C.c_int32)),
+                ("arrival", C.c_double), ("user_tag", C.c_uint64)]
+
+
+class Completion(C.Structure):
+    _fields_ = [("req_id", C.c_uint64), ("user_tag", C.c_uint64), ("t_arrival", C.c_double),
+                ("t_first", C.c_double), ("t_done", C.c_double)]
+
+
+class Result(C.Structure):
+    _fields_ = [("h", C.POINTER(C.c_float)), ("c", C.POINTER(C.c_float)),
+                ("tokens", C.POINTER(C.c_int32)), ("logits", C.POINTER(C.c_float))]
+
+
+class TaskRecord(C.Structure):
+    _fields_ = [("task", C.c_int), ("cell", C.c_int), ("tick", C.c_double),
+                ("first_row", C.c_int), ("n_rows", C.c_int)]
+
+
+class RowRecord(C.Structure):
+    _fields_ = [("req_id", C.c_uint64), ("node", C.c_int), ("slot", C.c_int)]
+
+
+class StepRow(C.Structure):
+    _fields_ = [("a", C.c_int32), ("b", C.c_int32), ("slot", C.c_int32), ("flags", C.c_int32)]
+
+
+class Stats(C.Structure):
+    _fields_ = [("tasks", C.c_uint64), ("rows", C.c_uint64), ("kernel_launches", C.c_uint64),
+                ("timed_launches", C.c_uint64), ("timed_ms", C.c_double),
+                ("timed_bytes", C.c_double), ("timed_flops", C.c_double),
+                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64)]
+
+
+# exported symbols (tests/test_abi.py checks them against include/bm.h)
+_P = C.c_void_p
+_SIGS = {
+    "bm_config_default": (None, [C.POINTER(Config)]),
+    "bm_create": (C.c_int, [C.POINTER(Config), C.POINTER(_P)]),
+    "bm_destroy": (None, [_P]),
+    "bm_strerror": (C.c_char_p, [C.c_int]),
+    "bm_abi_version": (C.c_int, []),
+    "bm_load_cell": (C.c_int, [_P, C.POINTER(CellDesc), C.POINTER(Weights), C.POINTER(C.c_int)]),
+    "bm_submit": (C.c_int, [_P, C.POINTER(Request), C.POINTER(C.c_uint64)]),
+    "bm_schedule_step": (C.c_int, [_P, C.POINTER(C.c_int)]),
+    "bm_poll": (C.c_int, [_P, C.POINTER(Completion), C.c_int, C.POINTER(C.c_int)]),
+    "bm_run": (C.c_int, [_P, C.POINTER(C.c_int)]),
+    "bm_read_result": (C.c_int, [_P, C.c_uint64, C.POINTER(Result)]),
+    "bm_release": (C.c_int, [_P, C.c_uint64]),
+    "bm_read_log": (C.c_int, [_P, C.POINTER(TaskRecord), C.c_int, C.POINTER(C.c_int)]),
+    "bm_read_log_rows": (C.c_int, [_P, C.POINTER(RowRecord), C.c_int, C.POINTER(C.c_int)]),
+    "bm_cell_step": (C.c_int, [_P, C.c_int, C.POINTER(StepRow), C.c_int, C.c_int]),
+    "bm_pool_write": (C.c_int, [_P, C.c_int, C.c_int, C.POINTER(C.c_int32), C.c_int,
+                                C.POINTER(C.c_float), C.POINTER(C.c_float)]),
+    "bm_pool_read": (C.c_int, [_P, C.c_int, C.c_int, C.POINTER(C.c_int32), C.c_int,
+                               C.POINTER(C.c_float), C.POINTER(C.c_float)]),
+    "bm_result_rows": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_int, C.POINTER(C.c_float),
+                                 C.POINTER(C.c_float)]),
+    "bm_tokens": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_int, C.POINTER(C.c_int32), C.c_int]),
+    "bm_get_stats": (C.c_int, [_P, C.POINTER(Stats)]),
+    "bm_reset_stats": (C.c_int, [_P]),
+    "bm_stream": (C.c_void_p, [_P]),
+}
+for _name, (_res, _args) in _SIGS.items():
+    _f = getattr(lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+
+class BMError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: {lib.bm_strerror(status).decode()} ({status})")
+
+
+def _ck(status: int, where: str) -> int:
+    if status != OK:
+        raise BMError(status, where)
+    return status
+
+
+def _f32(a) -> np.ndarray:
+    return np.ascontiguousarray(a, dtype=np.float32)
+
+
+def _i32(a) -> np.ndarray:
+    return np.ascontiguousarray(a, dtype=np.int32)
+
+
+def _fp(a: Optional[np.ndarray]):
+    return None if a is None else a.ctypes.data_as(C.POINTER(C.c_float))
+
+
+def _ip(a: Optional[np.ndarray]):
+    return None if a is None else a.ctypes.data_as(C.POINTER(C.c_int32))
+
+
+def default_config(**kw) -> Config:
+    cfg = Config()
+    lib.bm_config_default(C.byref(cfg))
+    for k, v in kw.items():
+        setattr(cfg, k, int(v))
+    return cfg
+
+
+class Engine:
+    """One engine per GPU (include/bm.h). Methods mirror the C entry points one to one."""
+
+    def __init__(self, **cfg):
+        self.cfg = default_config(**cfg)
+        h = C.c_void_p()
+        _ck(lib.bm_create(C.byref(self.cfg), C.byref(h)), "bm_create")
+        self.h = h
+        self._keep = []
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.bm_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ---------------------------------------------------------------- cells
+    def load_cell(self, kind: int, layers: int, vocab: int, max_batch: int, priority: int,
+                  W: Sequence[np.ndarray], b: Sequence[np.ndarray], E: Optional[np.ndarray] = None,
+                  W_out: Optional[np.ndarray] = None, b_out: Optional[np.ndarray] = None) -> int:
+        d = CellDesc(kind, self.cfg.hidden, layers, vocab, max_batch, priority)
+        Ws = [_f32(x) for x in W]
+        bs = [_f32(x) for x in b]
+        Wa = (C.POINTER(C.c_float) * len(Ws))(*[_fp(x) for x in Ws])
+        ba = (C.POINTER(C.c_float) * len(bs))(*[_fp(x) for x in bs])
+        Ea = _f32(E) if E is not None else None
+        Wo = _f32(W_out) if W_out is not None else None
+        bo = _f32(b_out) if b_out is not None else None
+        w = Weights(Wa, ba, _fp(Ea), _fp(Wo), _fp(bo))
+        cid = C.c_int()
+        _ck(lib.bm_load_cell(self.h, C.byref(d), C.byref(w), C.byref(cid)), "bm_load_cell")
+        return cid.value
+
+    # ---------------------------------------------------------------- requests
+    def submit(self, kind: int, cell0: int, cell1: int, tokens, arrival: float = 0.0,
+               decode_len: int = 0, left=None, right=None, tag: int = 0) -> int:
+        t = _i32(tokens)
+        l = _i32(left) if left is not None else None
+        r = _i32(right) if right is not None else None
+        q = Request(kind, cell0, cell1, len(t), _ip(t), decode_len, _ip(l), _ip(r),
+                    float(arrival), tag)
+        rid = C.c_uint64()
+        _ck(lib.bm_submit(self.h, C.byref(q), C.byref(rid)), "bm_submit")
+        return rid.value
+
+    def schedule_step(self) -> int:
+        n = C.c_int()
+        s = lib.bm_schedule_step(self.h, C.byref(n))
+        if s == E_AGAIN:
+            return -1
+        _ck(s, "bm_schedule_step")
+        return n.value
+
+    def poll(self, cap: int = 1 << 16) -> List[Completion]:
+        buf = (Completion * cap)()
+        n = C.c_int()
+        _ck(lib.bm_poll(self.h, buf, cap, C.byref(n)), "bm_poll")
+        return [buf[i] for i in range(n.value)]
+
+    def run(self) -> int:
+        n = C.c_int()
+        _ck(lib.bm_run(self.h, C.byref(n)), "bm_run")
+        return n.value
+
+    def read_result(self, rid: int, layers: int, decode_len: int = 0, vocab: int = 0):
+        H = self.cfg.hidden
+        h = np.zeros((layers, H), np.float32)
+        c = np.zeros((layers, H), np.float32)
+        L = self.cfg.pool_layers
+        hh = np.zeros((L, H), np.float32)
+        cc = np.zeros((L, H), np.float32)
+        toks = np.zeros(max(decode_len, 1), np.int32)
+        lg = np.zeros((max(decode_len, 1), vocab), np.float32) if vocab else None
+        res = Result(_fp(hh), _fp(cc), _ip(toks), _fp(lg))
+        _ck(lib.bm_read_result(self.h, rid, C.byref(res)), "bm_read_result")
+        h[:] = hh[:layers]
+        c[:] = cc[:layers]
+        return {"h": h, "c": c, "tokens": toks[:decode_len], "logits": lg}
+
+    def release(self, rid: int):
+        _ck(lib.bm_release(self.h, rid), "bm_release")
+
+    def read_log(self):
+        n = C.c_int()
+        _ck(lib.bm_read_log(self.h, None, 0, C.byref(n)), "bm_read_log")
+        tasks = (TaskRecord * max(n.value, 1))()
+        _ck(lib.bm_read_log(self.h, tasks, n.value, C.byref(n)), "bm_read_log")
+        m = C.c_int()
+        _ck(lib.bm_read_log_rows(self.h, None, 0, C.byref(m)), "bm_read_log_rows")
+        rows = (RowRecord * max(m.value, 1))()
+        _ck(lib.bm_read_log_rows(self.h, rows, m.value, C.byref(m)), "bm_read_log_rows")
+        out = []
+        for i in range(n.value):
+            t = tasks[i]
+            rr = [(int(rows[j].req_id), rows[j].node, rows[j].slot)
+                  for j in range(t.first_row, t.first_row + t.n_rows)]
+            out.append({"task": t.task, "cell": t.cell, "tick": t.tick, "rows": rr})
+        return out
+
+    # ---------------------------------------------------------------- direct cell access
+    def cell_step(self, cell: int, rows, sync: bool = True):
+        """rows: int32 array [b, 4] = (a, b, slot, flags) per bm_step_row."""
+        r = _i32(rows).reshape(-1, 4)
+        arr = (StepRow * len(r)).from_buffer_copy(r.tobytes())
+        _ck(lib.bm_cell_step(self.h, cell, arr, len(r), 0 if sync else 1), "bm_cell_step")
+
+    def pool_write(self, layer: int, parity: int, slots, h=None, c=None):
+        s = _i32(slots)
+        hh = _f32(h) if h is not None else None
+        cc = _f32(c) if c is not None else None
+        _ck(lib.bm_pool_write(self.h, layer, parity, _ip(s), len(s), _fp(hh), _fp(cc)), "bm_pool_write")
+
+    def pool_read(self, layer: int, parity: int, slots):
+        s = _i32(slots)
+        H = self.cfg.hidden
+        h = np.zeros((len(s), H), np.float32)
+        c = np.zeros((len(s), H), np.float32)
+        _ck(lib.bm_pool_read(self.h, layer, parity, _ip(s), len(s), _fp(h), _fp(c)), "bm_pool_read")
+        return h, c
+
+    def result_rows(self, idx):
+        i = _i32(idx)
+        LH = self.cfg.hidden * self.cfg.pool_layers
+        h = np.zeros((len(i), self.cfg.pool_layers, self.cfg.hidden), np.float32)
+        c = np.zeros_like(h)
+        _ck(lib.bm_result_rows(self.h, _ip(i), len(i), _fp(h), _fp(c)), "bm_result_rows")
+        return h, c
+
+    def tokens(self, slots, values=None):
+        s = _i32(slots)
+        v = _i32(values) if values is not None else np.zeros(len(s), np.int32)
+        _ck(lib.bm_tokens(self.h, _ip(s), len(s), _ip(v), 1 if values is not None else 0), "bm_tokens")
+        return v
+
+    def stats(self) -> dict:
+        st = Stats()
+        _ck(lib.bm_get_stats(self.h, C.byref(st)), "bm_get_stats")
+        return {k: getattr(st, k) for k, _ in Stats._fields_}
+
+    def reset_stats(self):
+        _ck(lib.bm_reset_stats(self.h), "bm_reset_stats")
+
+    def stream(self) -> int:
+        return int(lib.bm_stream(self.h) or 0)

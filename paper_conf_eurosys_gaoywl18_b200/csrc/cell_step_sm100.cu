@@ -1,0 +1,514 @@
+// cell_step_sm100.cu -- the hot path of cellular batching on B200 (sm_100a).
+//
+// ONE kernel = one batched cell step (one layer of an LSTM stack, a TreeLSTM leaf or internal
+// step, or the Seq2Seq output projection + argmax) over a dynamically assembled set of rows
+// that sit at different steps of different requests (§3.1-§3.2):
+//
+//   gather by slot (A6)  ->  [x ; h] . W^T on tcgen05 (A8)  ->  fused gates + state update
+//   + scatter back to the pool by slot (A9)           (projection: + argmax, A10)
+//
+// The paper copies the batch into contiguous buffers ("gather", §4.3) and runs MXNet
+// operators (cuBLAS GEMM + elementwise kernels) per cell. Here the gather is the operand load
+// of the GEMM itself and the elementwise work is the GEMM's epilogue.
+//
+// Orientation ("swap-AB"): the tensor-core M dimension is the weight rows (gate outputs), the
+// N dimension is the batch. A = packed weights (TMA, 128B swizzle), B = gathered activations
+// (cp.async, 128B swizzle written by hand), D = fp32 accumulators in TMEM (lane = weight row,
+// column = batch row).
+//
+// Grid = (S, H/U, ceil(b/256)); cluster = (S, 1, 1). The S CTAs of a cluster split K (the
+// [x ; h] width 2h) into S slices of `kslice` and reduce their fp32 partial tiles through
+// distributed shared memory in a FIXED order (s = 0..S-1), so the result of a row does not
+// depend on which other rows share the task (batch invariance, P10).
+//
+// Roles: warps 0-7 gather the activation tile (and lane 0 of warp 0 issues the weight TMA);
+// warp 8 allocates TMEM and issues tcgen05.mma from one lane. After the main loop warps 0-7
+// move the accumulators TMEM -> smem, the cluster reduces, and warps 0-7 run the epilogue.
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#include "kernels.h"
+
+namespace bm {
+namespace {
+
+constexpr int kStages = 4;
+constexpr int kBK = 64;                 // K elements per stage (128 B of bf16 = one SW128 atom)
+constexpr int kProducerThreads = 256;   // warps 0-7
+constexpr int kThreads = kProducerThreads + 32;
+constexpr int kMaxCols = 256;           // batch columns per CTA (MMA N <= 256)
+constexpr int kWStageBytes = 128 * 128; // 128 weight rows x 128 B
+constexpr int kLag = 2;                 // cp.async groups in flight per producer thread
+
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(bar), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  while (!mbar_try_wait(bar, parity)) {
+  }
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar,
+                                            int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void cp_async_16(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
+               "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
+                   : "memory");
+}
+__device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ float4 ld_cluster_v4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(addr)
+               : "memory");
+  return v;
+}
+
+// UMMA shared-memory descriptor: K-major, 128B swizzle, 8-row groups 1024 B apart (SBO).
+__device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= static_cast<uint64_t>((saddr >> 4) & 0x3FFF);
+  d |= static_cast<uint64_t>(1) << 16;            // LBO (unused for swizzled K-major)
+  d |= static_cast<uint64_t>(1024 >> 4) << 32;    // SBO
+  d |= static_cast<uint64_t>(1) << 46;            // descriptor version (sm_100)
+  d |= static_cast<uint64_t>(2) << 61;            // SWIZZLE_128B
+  return d;
+}
+// Instruction descriptor, kind::f16: D fp32, A bf16, B bf16, both K-major, M x N.
+__device__ __forceinline__ uint32_t idesc_bf16(int M, int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(N >> 3) << 17) |
+         (static_cast<uint32_t>(M >> 4) << 24);
+}
+__device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc,
+                                         uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void mma_commit(uint32_t bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar)
+      : "memory");
+}
+// 32 lanes x 32 columns of fp32 from TMEM into registers (one column per register).
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
+  uint32_t r[32];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, "
+      "%11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, "
+      "%28, %29, %30, %31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
+        "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
+        "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
+        "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+__device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
+
+// ------------------------------------------------------------------ row sources (A6)
+// Pointer to the first element of a row's operand segment `seg`, or nullptr for a zero row.
+template <int EPI>
+__device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const RowDesc& r,
+                                                        int seg) {
+  const size_t H = p.H;
+  const size_t S = p.n_slots;
+  const __nv_bfloat16* hp = static_cast<const __nv_bfloat16*>(p.h_pool);
+  if constexpr (EPI == EPI_LSTM) {
+    const int par = (r.flags & ROW_PARITY) ? 1 : 0;
+    if (seg == 0) {
+      if (p.h_lower != nullptr) {  // layer > 0: x = h'(layer-1) just written at parity 1-par
+        return static_cast<const __nv_bfloat16*>(p.h_lower) + ((1 - par) * S + r.slot) * H;
+      }
+      const int tok = r.a >= 0 ? r.a : p.tok[r.slot];
+      return static_cast<const __nv_bfloat16*>(p.E) + static_cast<size_t>(tok) * H;
+    }
+    if (r.flags & ROW_FIRST) return nullptr;  // h_prev = 0
+    return hp + (par * S + r.slot) * H;
+  } else if constexpr (EPI == EPI_LEAF) {
+    return static_cast<const __nv_bfloat16*>(p.E) + static_cast<size_t>(r.a) * H;
+  } else if constexpr (EPI == EPI_INTERNAL) {
+    return hp + static_cast<size_t>(seg == 0 ? r.a : r.b) * H;  // children h at parity 0
+  } else {  // EPI_PROJ: h of the top layer, written at parity 1-par by this step
+    const int par = (r.flags & ROW_PARITY) ? 1 : 0;
+    return hp + ((1 - par) * S + r.slot) * H;
+  }
+}
+
+// ------------------------------------------------------------------ the kernel
+template <int EPI>
+__global__ void __launch_bounds__(kThreads, 1)
+    cell_step_sm100_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ StepArgs p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5;
+  const int lane = tid & 31;
+  const int G = EPI == EPI_PROJ ? 1 : gates_of(EPI);
+  const int U = p.U;
+  const int tile_rows = EPI == EPI_PROJ ? 128 : G * U;
+  const uint32_t rank = (EPI == EPI_PROJ) ? 0u : cluster_rank();
+  const int col0 = blockIdx.z * kMaxCols;
+  const int ncols = min(kMaxCols, p.b - col0);
+  const int npad = (ncols + 15) & ~15;
+  const int nk = p.kslice / kBK;
+  const int k_begin = static_cast<int>(rank) * p.kslice;
+
+  // shared memory carve-up
+  uint8_t* w_st = smem;                                   // kStages x 16 KB
+  uint8_t* x_st = smem + kStages * kWStageBytes;          // kStages x npad x 128 B
+  const int x_stage_bytes = npad * 128;
+  uint8_t* tail = x_st + kStages * x_stage_bytes;
+  const __nv_bfloat16** src_tab = reinterpret_cast<const __nv_bfloat16**>(tail);  // [2][256]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(tail + 2 * kMaxCols * sizeof(void*));
+  const uint32_t full0 = smem_u32(bars);
+  const uint32_t empty0 = smem_u32(bars + kStages);
+  const uint32_t done_bar = smem_u32(bars + 2 * kStages);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kStages + 1);
+  int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
+
+  // ---- setup
+  if (tid == 0) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(full0 + 8 * s, kProducerThreads);
+      mbar_init(empty0 + 8 * s, 1);
+    }
+    mbar_init(done_bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+  }
+  if (warp == 8) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "r"(256)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  for (int c = tid; c < kMaxCols; c += kThreads) {
+    const __nv_bfloat16* s0 = nullptr;
+    const __nv_bfloat16* s1 = nullptr;
+    if (c < ncols) {
+      const RowDesc r = p.rows[col0 + c];
+      s0 = seg_src<EPI>(p, r, 0);
+      if (p.K1 > 0) s1 = seg_src<EPI>(p, r, 1);
+    }
+    src_tab[c] = s0;
+    src_tab[kMaxCols + c] = s1;
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp < 8) {
+    // ================================================================ producers (A6, A7)
+    const __nv_bfloat16* dummy = static_cast<const __nv_bfloat16*>(p.E != nullptr ? p.E : p.h_pool);
+    const int wbytes = tile_rows * 128;
+    const int wrow0 = blockIdx.y * tile_rows;
+    for (int kb = 0; kb < nk; ++kb) {
+      const int s = kb % kStages;
+      const int round = kb / kStages;
+      if (round > 0) mbar_wait(empty0 + 8 * s, (round - 1) & 1);
+      const int k = k_begin + kb * kBK;
+      const int seg = k >= p.K0 ? 1 : 0;
+      const int kk = k - seg * p.K0;
+      if (tid == 0) {
+        mbar_expect_tx(full0 + 8 * s, wbytes);
+        tma_load_2d(smem_u32(w_st + s * kWStageBytes), &tmW, full0 + 8 * s, k, wrow0);
+      }
+      const uint32_t xs = smem_u32(x_st + s * x_stage_bytes);
+      const __nv_bfloat16** tab = src_tab + seg * kMaxCols;
+      for (int q = tid; q < npad * 8; q += kProducerThreads) {
+        const int row = q >> 3;
+        const int ch = q & 7;
+        const __nv_bfloat16* src = tab[row];
+        const uint32_t dst = xs + row * 128 + ((ch ^ (row & 7)) << 4);
+        if (src != nullptr) {
+          cp_async_16(dst, src + kk + ch * 8, 16);
+        } else {
+          cp_async_16(dst, dummy, 0);  // zero fill
+        }
+      }
+      cp_async_commit();
+      if (kb >= kLag) {
+        cp_async_wait<kLag>();
+        fence_proxy_async();
+        mbar_arrive(full0 + 8 * ((kb - kLag) % kStages));
+      }
+    }
+    cp_async_wait<0>();
+    fence_proxy_async();
+    for (int kb = max(0, nk - kLag); kb < nk; ++kb) mbar_arrive(full0 + 8 * (kb % kStages));
+  } else {
+    // ================================================================ MMA issuer (A8)
+    const uint32_t idesc = idesc_bf16(128, npad);
+    for (int kb = 0; kb < nk; ++kb) {
+      const int s = kb % kStages;
+      mbar_wait(full0 + 8 * s, (kb / kStages) & 1);
+      tc_fence_after();
+      if (lane == 0) {
+        const uint64_t a = sdesc_sw128(smem_u32(w_st + s * kWStageBytes));
+        const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes));
+#pragma unroll
+        for (int k = 0; k < kBK / 16; ++k) {
+          mma_bf16(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
+        }
+        mma_commit(empty0 + 8 * s);
+        if (kb == nk - 1) mma_commit(done_bar);
+      }
+      __syncwarp();
+    }
+  }
+
+  // ================================================================ accumulators -> smem
+  float* P = reinterpret_cast<float*>(smem);  // reuses the (drained) stage buffers
+  const int pitch = EPI == EPI_PROJ ? 129 : 128;
+  if (warp < 8) {
+    mbar_wait(done_bar, 0);
+    tc_fence_after();
+    const int q = warp & 3;
+    const int row = 32 * q + lane;
+    for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
+      float v[32];
+      tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        if (c0 + i < npad) P[(c0 + i) * pitch + row] = v[i];
+      }
+    }
+  }
+  tc_fence_before();
+
+  if constexpr (EPI == EPI_PROJ) {
+    // ============================================================ projection + argmax (A10)
+    __syncthreads();
+    const int v0 = blockIdx.y * 128;
+    for (int c = tid; c < ncols; c += kThreads) {
+      const RowDesc r = p.rows[col0 + c];
+      float best = -INFINITY;
+      int besti = 0;
+      float* lg = nullptr;
+      if (p.logits != nullptr) {
+        lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + r.b) * p.V + v0;
+      }
+      for (int i = 0; i < 128; ++i) {
+        const float z = P[c * pitch + i] + p.bias[v0 + i];
+        if (lg != nullptr) lg[i] = z;
+        if (z > best) {  // strict: keeps the lowest index among equal maxima
+          best = z;
+          besti = i;
+        }
+      }
+      uint32_t ob = __float_as_uint(best);
+      ob = (ob & 0x80000000u) ? ~ob : (ob | 0x80000000u);
+      const unsigned long long key =
+          (static_cast<unsigned long long>(ob) << 32) | (0xFFFFFFFFu - static_cast<uint32_t>(v0 + besti));
+      atomicMax(p.amax + col0 + c, key);
+    }
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) {
+      const unsigned total = gridDim.x * gridDim.y * gridDim.z;
+      const unsigned prev = atomicAdd(p.done_ctas, 1u);
+      *flag_last = (prev == total - 1) ? 1 : 0;
+    }
+    __syncthreads();
+    if (*flag_last) {  // last CTA: publish argmax -> feed token + emitted token, reset keys
+      __threadfence();
+      for (int c = tid; c < p.b; c += kThreads) {
+        const RowDesc r = p.rows[c];
+        const unsigned long long key = atomicExch(p.amax + c, 0ull);
+        const int y = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(key & 0xFFFFFFFFull));
+        p.tok[r.slot] = y;
+        p.res_tok[static_cast<size_t>(r.flags >> 8) * p.max_decode + r.b] = y;
+      }
+      if (tid == 0) *p.done_ctas = 0;
+    }
+  } else {
+    // ============================================================ split-K reduction + gates (A9)
+    cluster_sync();
+    const int S = p.S;
+    uint32_t peer[8];
+    for (int s = 0; s < S; ++s) peer[s] = mapa(smem_u32(P), s);
+    const int cper = (ncols + S - 1) / S;
+    const int c_lo = static_cast<int>(rank) * cper;
+    const int c_hi = min(ncols, c_lo + cper);
+    const int unit0 = blockIdx.y * U;
+    const int prow0 = blockIdx.y * tile_rows;
+    const size_t H = p.H;
+    const size_t NS = p.n_slots;
+    if (warp < 8) {
+      const int cols_per_pass = kProducerThreads / U;
+      for (int c = c_lo + tid / U; c < c_hi; c += cols_per_pass) {
+        const int j = tid % U;
+        float z[5];
+#pragma unroll
+        for (int g = 0; g < 5; ++g) z[g] = 0.f;
+        const uint32_t off = static_cast<uint32_t>((c * pitch + j * G) * 4);
+        for (int s = 0; s < S; ++s) {  // fixed order -> deterministic, batch-invariant
+          if (G == 4) {
+            const float4 v = ld_cluster_v4(peer[s] + off);
+            z[0] += v.x;
+            z[1] += v.y;
+            z[2] += v.z;
+            z[3] += v.w;
+          } else {
+#pragma unroll
+            for (int g = 0; g < 5; ++g)
+              if (g < G) z[g] += ld_cluster_f32(peer[s] + off + 4 * g);
+          }
+        }
+#pragma unroll
+        for (int g = 0; g < 5; ++g)
+          if (g < G) z[g] += p.bias[prow0 + j * G + g];
+        const RowDesc r = p.rows[col0 + c];
+        const int u = unit0 + j;
+        float hn, cn;
+        if constexpr (EPI == EPI_LSTM) {
+          const float cp = (r.flags & ROW_FIRST) ? 0.f : p.c_pool[r.slot * H + u];
+          cn = sigm(z[1]) * cp + sigm(z[0]) * tanhf(z[2]);
+          hn = sigm(z[3]) * tanhf(cn);
+        } else if constexpr (EPI == EPI_LEAF) {
+          cn = sigm(z[0]) * tanhf(z[2]);
+          hn = sigm(z[1]) * tanhf(cn);
+        } else {
+          const float cl = p.c_pool[static_cast<size_t>(r.a) * H + u];
+          const float cr = p.c_pool[static_cast<size_t>(r.b) * H + u];
+          cn = sigm(z[0]) * tanhf(z[4]) + sigm(z[1]) * cl + sigm(z[2]) * cr;
+          hn = sigm(z[3]) * tanhf(cn);
+        }
+        p.c_pool[r.slot * H + u] = cn;
+        const int par_out = (EPI == EPI_LSTM) ? ((r.flags & ROW_PARITY) ? 0 : 1) : 0;
+        static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + r.slot) * H + u] = __float2bfloat16_rn(hn);
+        if (r.flags & ROW_LAST) {
+          const size_t ro = (static_cast<size_t>(r.flags >> 8) * p.res_layers + p.layer) * H + u;
+          p.res_h[ro] = hn;
+          p.res_c[ro] = cn;
+        }
+      }
+    }
+    cluster_sync();  // peers may still read this CTA's partials until here
+  }
+
+  if (warp == 8) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256)
+                 : "memory");
+  }
+}
+
+template <int EPI>
+cudaError_t launch_impl(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t st) {
+  const int cols = a.b < kMaxCols ? a.b : kMaxCols;
+  const int npad = (cols + 15) & ~15;
+  const size_t smem = 1024 + kStages * (kWStageBytes + npad * 128) + 2 * kMaxCols * sizeof(void*) +
+                      (2 * kStages + 1) * 8 + 16;
+  static bool configured = false;
+  if (!configured) {
+    cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         1024 + kStages * (kWStageBytes + kMaxCols * 128) +
+                                             2 * kMaxCols * (int)sizeof(void*) + (2 * kStages + 1) * 8 + 16);
+    if (e != cudaSuccess) return e;
+    configured = true;
+  }
+  const int S = EPI == EPI_PROJ ? 1 : a.S;
+  const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(S, tiles, (a.b + kMaxCols - 1) / kMaxCols);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = S;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI>, tmW, a);
+}
+
+}  // namespace
+
+cudaError_t launch_cell_step_sm100(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t st) {
+  if (a.b <= 0) return cudaSuccess;
+  switch (a.epi) {
+    case EPI_LSTM: return launch_impl<EPI_LSTM>(a, tmW, st);
+    case EPI_LEAF: return launch_impl<EPI_LEAF>(a, tmW, st);
+    case EPI_INTERNAL: return launch_impl<EPI_INTERNAL>(a, tmW, st);
+    case EPI_PROJ: return launch_impl<EPI_PROJ>(a, tmW, st);
+  }
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace bm

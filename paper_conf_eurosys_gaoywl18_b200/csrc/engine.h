@@ -1,0 +1,166 @@
+// engine.h -- internal structures of the host runtime behind include/bm.h.
+//
+//   Engine
+//    ├─ cells[]        loaded cell types: packed device weights + TMA maps + scheduler queue
+//    ├─ reqs[]         request table (ring of max_requests entries): cell graph + subgraphs
+//    ├─ SlotPool       lowest-free-index allocator over the HBM state pool (A4)
+//    ├─ Scheduler      Algorithm 1 (Schedule / Batch / FormBatchedTask)
+//    ├─ in-flight FIFO tasks launched, not yet retired (the paper's in-progress queue, L331)
+//    └─ device         pool h/c, feed tokens, result rows, row-descriptor ring, signal counter
+#pragma once
+#include <stdint.h>
+
+#include <chrono>
+#include <deque>
+#include <string>
+#include <vector>
+
+#include "../../include/bm.h"
+#include "kernels.h"
+
+namespace bm {
+
+struct Engine;
+
+// ---------------------------------------------------------------- cell graph (A1, D1-D3)
+struct Subgraph {
+  int req = -1;            // request table index
+  int sid = 0;             // subgraph id within the request
+  int ct = 0;              // cell type
+  int n_nodes = 0;
+  int n_submitted = 0;
+  int n_completed = 0;
+  int pinned = -1;         // worker id or -1 (Alg. 1 line 21, L381)
+  int inflight = 0;        // tasks in flight holding nodes of this subgraph
+  std::vector<int> ready;  // ready, unsubmitted nodes, ascending (height, post-order index)
+  // intrusive FIFO links of the cell type's subgraph queue (D3)
+  int q_prev_req = -1, q_prev_sid = -1, q_next_req = -1, q_next_sid = -1;
+  bool queued = false;
+};
+
+struct Request {
+  bool used = false;
+  bool done = false;
+  uint64_t id = 0;          // admission index
+  uint64_t tag = 0;
+  int kind = 0;
+  int cell0 = 0, cell1 = 0;
+  int n_nodes = 0;          // chain: L; seq2seq: S + T; tree: n
+  int enc_len = 0;          // seq2seq: S
+  int n_completed = 0;
+  int leaves_left = 0;
+  int internal_sid = -1;
+  bool started = false;     // slots taken
+  int slot = -1;            // chain / seq2seq
+  double t_arrival = 0, t_first = -1, t_done = -1;
+  std::vector<int32_t> tokens;      // chain/seq2seq: source tokens; tree: per node
+  std::vector<int32_t> left, right, parent, height, node_slot;
+  std::vector<uint8_t> submitted;
+  std::vector<Subgraph> sg;
+  std::vector<int> node_sid;        // trees: subgraph of each node
+};
+
+struct Cell {
+  bm_cell_desc d{};
+  int epi = 0, G = 0, U = 0, S = 1, kslice = 0, K0 = 0, K1 = 0;
+  // device weights (per layer for LSTM stacks)
+  std::vector<void*> W;
+  std::vector<float*> bias;
+  std::vector<CUtensorMap> tm;
+  void* E = nullptr;
+  void* W_out = nullptr;
+  float* b_out = nullptr;
+  CUtensorMap tm_out{};
+  // scheduler state of this cell type
+  int q_head_req = -1, q_head_sid = -1, q_tail_req = -1, q_tail_sid = -1;
+  int64_t ready_nodes = 0;   // NumReadyNodes (S16)
+  int running_tasks = 0;     // NumRunningTasks (S17)
+};
+
+struct TaskRow {
+  int req;     // request table index
+  int node;
+  int slot;
+};
+
+struct Task {
+  uint64_t seq = 0;          // launch index
+  int ct = 0;
+  double tick = 0;           // submit time
+  double finish = 0;         // VIRTUAL: retire tick
+  int ring_off = 0;          // first row in the descriptor ring
+  int b = 0;
+  std::vector<TaskRow> rows;
+  int ev_first = -1, ev_count = 0;  // timed launches (time_kernels)
+};
+
+struct TimedLaunch {
+  cudaEvent_t beg, end;
+  double bytes, flops;
+};
+
+struct Engine {
+  bm_config cfg{};
+  bool sticky_cuda = false;
+  bool submitted_any = false;
+  std::vector<Cell> cells;
+  std::vector<Request> reqs;        // ring of max_requests
+  int n_live_reqs = 0;
+  uint64_t next_req_id = 0;
+  std::deque<int> pending;          // request table indices not yet admitted (FIFO, S21)
+  std::vector<int> free_slots_heap; // min-heap of free slots (A4)
+  std::deque<Task> inflight;        // in-progress queue (L331, L395)
+  uint64_t launched = 0;            // tasks launched so far (== signal target)
+  double now = 0;                   // clock: ticks (VIRTUAL/DRY) or seconds since bm_run
+  double last_finish = 0;
+  std::chrono::steady_clock::time_point t0;
+  bool wall_started = false;
+  std::vector<bm_completion> completions;   // not yet returned by bm_poll
+  std::vector<bm_task_record> log_tasks;
+  std::vector<bm_row_record> log_rows;
+  bm_stats stats{};
+
+  // ---- device
+  cudaStream_t stream = nullptr;
+  void* h_pool = nullptr;          // [layers][2][slots][H]
+  float* c_pool = nullptr;         // [layers][slots][H]
+  int* tok = nullptr;              // [slots]
+  float* res_h = nullptr;          // [max_requests][layers][H]
+  float* res_c = nullptr;
+  int32_t* res_tok = nullptr;      // [max_requests][max_decode]
+  float* logits = nullptr;         // [max_requests][max_decode][V] (record_logits)
+  int logits_vocab = 0;
+  unsigned long long* amax = nullptr;
+  unsigned int* done_ctas = nullptr;
+  RowDesc* ring_dev = nullptr;
+  RowDesc* ring_host = nullptr;    // pinned staging
+  int ring_rows = 0;
+  int ring_head = 0;               // next free row
+  int ring_used = 0;               // rows held by in-flight tasks
+  unsigned long long* signal_host = nullptr;   // pinned, mapped
+  unsigned long long* signal_dev = nullptr;
+  RowDesc* direct_rows = nullptr;  // bm_cell_step rows (device)
+  std::vector<TimedLaunch> ev_pool;
+  int ev_head = 0;
+
+  bool device() const { return cfg.clock != BM_CLOCK_DRY; }
+  size_t elem() const { return cfg.precision == BM_PREC_BF16 ? 2 : 4; }
+  size_t H() const { return static_cast<size_t>(cfg.hidden); }
+  void* h_layer(int l) const {
+    return static_cast<char*>(h_pool) + static_cast<size_t>(l) * 2 * cfg.max_slots * H() * elem();
+  }
+  float* c_layer(int l) const { return c_pool + static_cast<size_t>(l) * cfg.max_slots * H(); }
+};
+
+// scheduler.cpp
+bm_status admit_request(Engine& e, int ri);
+int schedule(Engine& e, std::vector<Task>& out);     // Schedule(worker 0): tasks formed
+void retire_task(Engine& e, Task& t);
+bool has_ready(const Engine& e);
+void slot_release(Engine& e, int s);
+
+// runtime.cpp
+bm_status launch_tasks(Engine& e, std::vector<Task>& tasks);
+double wall_now(const Engine& e);
+
+}  // namespace bm

@@ -1,0 +1,77 @@
+// Internal interface between the host runtime (engine.cpp) and the sm_100a kernels.
+// Not part of the public C-ABI (include/bm.h).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace bm {
+
+// One row of a batched cell task (== bm_step_row in include/bm.h).
+struct RowDesc {
+  int32_t a;      // LSTM/leaf: token id, or -1 = device feed token tok[slot]; internal: left slot
+  int32_t b;      // internal: right slot; decoder projection: decode step index
+  int32_t slot;   // output slot (LSTM: also the state read)
+  int32_t flags;  // ROW_* | result_index << 8
+};
+enum { ROW_FIRST = 1, ROW_LAST = 2, ROW_PARITY = 4 };
+
+// Epilogue kinds (template parameter of the kernels).
+enum { EPI_LSTM = 0, EPI_PROJ = 1, EPI_LEAF = 2, EPI_INTERNAL = 3 };
+
+// Gates per cell kind and the packed ("gate-interleaved") weight layout:
+//   packed row n = u * G + g  <->  paper row g * H + u   (u = hidden unit, g = gate)
+// so that one tile of U units holds every gate of its units (fused epilogue, A9).
+__host__ __device__ inline int gates_of(int epi) {
+  return epi == EPI_LSTM ? 4 : epi == EPI_LEAF ? 3 : epi == EPI_INTERNAL ? 5 : 1;
+}
+
+struct StepArgs {
+  int epi;          // EPI_*
+  int G;            // gates (4 LSTM, 3 leaf, 5 internal, 1 projection)
+  int H;            // hidden
+  int K0, K1;       // widths of the two operand segments ([x ; h] or [h_L ; h_R]); K1 may be 0
+  int U;            // hidden units per CTA tile (tile rows = G * U <= 128)
+  int S;            // split-K factor = cluster size
+  int kslice;       // K per CTA (multiple of 64)
+  int b;            // rows in the task
+  int layer;        // layer index inside the pool (0-based)
+  int n_slots;      // pool slots (stride between the two h parities)
+  const RowDesc* rows;
+  const void* E;        // embedding [V][H] (bf16 or fp32)
+  int V;
+  const void* h_lower;  // pool h of layer-1, base of parity 0 ([2][n_slots][H]); layer 0: null
+  void* h_pool;         // pool h of this layer ([2][n_slots][H])
+  float* c_pool;        // pool c of this layer ([n_slots][H])
+  int* tok;             // feed tokens [n_slots]
+  const void* W;        // packed weights [rows][K] (SIMT path; the bf16 path uses the TMA map)
+  const float* bias;    // packed bias [rows]
+  int W_rows;           // G * H (or V for the projection)
+  float* res_h;         // result rows [max_requests][res_layers][H]
+  float* res_c;
+  int res_layers;
+  // projection + argmax (EPI_PROJ)
+  unsigned long long* amax;   // [bmax] packed (value, ~index) keys, zero between tasks
+  unsigned int* done_ctas;    // CTA completion counter for the last-CTA finalize
+  int32_t* res_tok;           // [max_requests][max_decode]
+  int max_decode;
+  float* logits;              // debug [max_requests][max_decode][V] or null
+};
+
+// bf16 / tcgen05 path (cell_step_sm100.cu). tmW: TMA map of the packed bf16 weights.
+cudaError_t launch_cell_step_sm100(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t st);
+// fp32 / SIMT path (cell_step_simt.cu)
+cudaError_t launch_cell_step_simt(const StepArgs& a, cudaStream_t st);
+
+// Weight preparation (load time): fp32 paper layout -> packed, gate-interleaved, bf16 or fp32.
+cudaError_t launch_pack_rows(const float* src, void* dst, float* bias_dst, const float* bias_src,
+                             int G, int H, int K, int bf16, cudaStream_t st);
+cudaError_t launch_convert(const float* src, void* dst, size_t n, int bf16, cudaStream_t st);
+// Completion signal (A12): bump a host-mapped counter after everything before it in stream.
+cudaError_t launch_signal(unsigned long long* counter, cudaStream_t st);
+// Pool access helpers (tests): gather/scatter fp32 rows of h (bf16 or fp32) and c.
+cudaError_t launch_pool_io(void* h_pool, float* c_pool, const int32_t* slots, int n, int H,
+                           float* h_buf, float* c_buf, int write, int bf16, cudaStream_t st);
+
+// Kernel-count bookkeeping: number of kernels one launch_* call issues.
+}  // namespace bm

@@ -1,0 +1,879 @@
+// runtime.cpp -- device side of the engine and the extern "C" entry points of include/bm.h.
+//
+// Launch path (A5, §5 "Keeping the GPU busy", L391): every task of one Schedule call is
+// staged in a pinned host ring of 16-byte row descriptors, copied to the device with ONE
+// cudaMemcpyAsync, and all kernels of all tasks are pushed onto one stream in order, without
+// waiting. After each task a signal kernel bumps a counter in mapped pinned host memory
+// (§5 "Asynchronous Completion Notification", L393-L395); bm_poll / the run loop compare the
+// counter against the in-progress FIFO and retire finished tasks in order.
+#include <cuda_bf16.h>
+#include <string.h>
+
+#include <algorithm>
+#include <functional>
+#include <new>
+#include <thread>
+
+#include "engine.h"
+
+namespace bm {
+
+double wall_now(const Engine& e) {
+  return std::chrono::duration<double>(std::chrono::steady_clock::now() - e.t0).count();
+}
+
+namespace {
+
+#define CK(x)                         \
+  do {                                \
+    cudaError_t err__ = (x);          \
+    if (err__ != cudaSuccess) {       \
+      e.sticky_cuda = true;           \
+      return BM_E_CUDA;               \
+    }                                 \
+  } while (0)
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  if (fn == nullptr) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  return fn;
+}
+
+// TMA map of a packed bf16 matrix [rows][K], box = 64 K-elements x box_rows, 128B swizzle.
+bool make_tmap(CUtensorMap* m, const void* base, int rows, int K, int box_rows) {
+  EncodeTiledFn fn = encode_fn();
+  if (fn == nullptr) return false;
+  cuuint64_t dims[2] = {static_cast<cuuint64_t>(K), static_cast<cuuint64_t>(rows)};
+  cuuint64_t strides[1] = {static_cast<cuuint64_t>(K) * 2};
+  cuuint32_t box[2] = {64, static_cast<cuuint32_t>(box_rows)};
+  cuuint32_t es[2] = {1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <class T>
+cudaError_t dalloc(T** p, size_t n) {
+  return cudaMalloc(reinterpret_cast<void**>(p), n * sizeof(T));
+}
+
+// Algorithmic bytes / flops of one cell-step launch: weights streamed
+// once, gathered operand rows, state read/written, result rows. Padding is not counted.
+void algo_cost(const Engine& e, const Cell& c, int b, bool proj, double* bytes, double* flops) {
+  const double H = static_cast<double>(e.cfg.hidden);
+  const double el = static_cast<double>(e.elem());
+  if (proj) {
+    const double V = c.d.vocab;
+    *bytes = V * H * el + V * 4 + b * (H * el + 8.0);
+    *flops = 2.0 * b * H * V;
+    return;
+  }
+  const double K = c.K0 + c.K1;
+  const double rows = static_cast<double>(c.G) * H;
+  double per_row = K * el + H * el + H * 4;              // gather, h' write, c' write
+  if (c.epi == EPI_LSTM) per_row += H * 4;                // c read
+  if (c.epi == EPI_INTERNAL) per_row += 2 * H * 4;        // c_L, c_R read
+  *bytes = rows * K * el + rows * 4 + b * per_row;
+  *flops = 2.0 * b * K * rows;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------- launching tasks
+static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, int b, int layer,
+                                 bool proj, int* ev_out) {
+  StepArgs a{};
+  a.epi = proj ? EPI_PROJ : c.epi;
+  a.G = proj ? 1 : c.G;
+  a.H = e.cfg.hidden;
+  a.K0 = c.K0;
+  a.K1 = proj ? 0 : c.K1;
+  a.U = c.U;
+  a.S = proj ? 1 : c.S;
+  a.kslice = proj ? e.cfg.hidden : c.kslice;
+  if (proj) {
+    a.S = 1;
+    a.kslice = e.cfg.hidden;
+  }
+  a.b = b;
+  a.layer = layer;
+  a.n_slots = e.cfg.max_slots;
+  a.rows = rows_dev;
+  a.E = c.E;
+  a.V = c.d.vocab;
+  const bool tree = c.epi == EPI_LEAF || c.epi == EPI_INTERNAL;
+  const int pl = tree ? 0 : (proj ? c.d.layers - 1 : layer);
+  a.h_lower = (!tree && !proj && layer > 0) ? e.h_layer(layer - 1) : nullptr;
+  a.h_pool = e.h_layer(pl);
+  a.c_pool = e.c_layer(pl);
+  a.tok = e.tok;
+  a.W = proj ? c.W_out : c.W[layer];
+  a.bias = proj ? c.b_out : c.bias[layer];
+  a.W_rows = proj ? c.d.vocab : c.G * e.cfg.hidden;
+  a.res_h = e.res_h;
+  a.res_c = e.res_c;
+  a.res_layers = e.cfg.pool_layers;
+  a.amax = e.amax;
+  a.done_ctas = e.done_ctas;
+  a.res_tok = e.res_tok;
+  a.max_decode = e.cfg.max_decode_len;
+  a.logits = (proj && e.logits != nullptr) ? e.logits : nullptr;
+  TimedLaunch* tl = nullptr;
+  if (e.cfg.time_kernels && !e.ev_pool.empty()) {
+    const int i = e.ev_head;
+    e.ev_head = (e.ev_head + 1) % static_cast<int>(e.ev_pool.size());
+    tl = &e.ev_pool[i];
+    algo_cost(e, c, b, proj, &tl->bytes, &tl->flops);
+    CK(cudaEventRecord(tl->beg, e.stream));
+    if (ev_out) *ev_out = i;
+  }
+  cudaError_t err;
+  if (e.cfg.precision == BM_PREC_BF16) err = launch_cell_step_sm100(a, proj ? c.tm_out : c.tm[layer], e.stream);
+  else err = launch_cell_step_simt(a, e.stream);
+  CK(err);
+  if (tl) CK(cudaEventRecord(tl->end, e.stream));
+  e.stats.kernel_launches += 1;
+  return BM_OK;
+}
+
+static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, int b, Task* t) {
+  const bool lstm = c.epi == EPI_LSTM;
+  const int L = lstm ? c.d.layers : 1;
+  for (int l = 0; l < L; ++l) {
+    int ev = -1;
+    bm_status s = launch_one_step(e, c, rows_dev, b, l, false, &ev);
+    if (s != BM_OK) return s;
+    if (t && ev >= 0) {
+      if (t->ev_first < 0) t->ev_first = ev;
+      t->ev_count += 1;
+    }
+  }
+  if (c.d.kind == BM_CELL_LSTM_PROJ) {
+    int ev = -1;
+    bm_status s = launch_one_step(e, c, rows_dev, b, 0, true, &ev);
+    if (s != BM_OK) return s;
+    if (t && ev >= 0) t->ev_count += 1;
+  }
+  return BM_OK;
+}
+
+// Row descriptor of a scheduled node (A3): what the kernels need to gather and scatter.
+static RowDesc make_row(const Engine& e, const Cell& c, const TaskRow& tr) {
+  const Request& r = e.reqs[tr.req];
+  RowDesc d{};
+  d.slot = tr.slot;
+  int flags = 0;
+  const int res = tr.req;  // result row = request table index
+  if (r.kind == BM_REQ_TREE) {
+    if (r.left[tr.node] < 0) {
+      d.a = r.tokens[tr.node];
+    } else {
+      d.a = r.node_slot[r.left[tr.node]];
+      d.b = r.node_slot[r.right[tr.node]];
+    }
+    if (tr.node == r.n_nodes - 1) flags |= ROW_LAST;
+  } else {
+    const int step = tr.node;  // global step (encoder steps then decoder steps)
+    if (step == 0) flags |= ROW_FIRST;
+    if (step & 1) flags |= ROW_PARITY;
+    if (r.kind == BM_REQ_CHAIN || step < r.enc_len) {
+      d.a = r.tokens[step];
+    } else {
+      const int s = step - r.enc_len;
+      d.a = s == 0 ? 1 /* <go> */ : -1 /* feed previous: tok[slot] on device */;
+      d.b = s;
+    }
+    if (step == r.n_nodes - 1) flags |= ROW_LAST;
+  }
+  (void)c;
+  d.flags = flags | (res << 8);
+  return d;
+}
+
+bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
+  if (tasks.empty()) return BM_OK;
+  int total = 0;
+  for (Task& t : tasks) total += static_cast<int>(t.rows.size());
+  for (Task& t : tasks) {
+    t.seq = e.launched++;
+    t.b = static_cast<int>(t.rows.size());
+    e.stats.tasks += 1;
+    e.stats.rows += t.b;
+    if (e.cfg.clock != BM_CLOCK_WALL) {
+      const double start = std::max(e.now, e.last_finish);
+      t.finish = start + 1.0;
+      e.last_finish = t.finish;
+    }
+    bm_task_record rec;
+    rec.task = static_cast<int>(t.seq);
+    rec.cell = t.ct;
+    rec.tick = t.tick;
+    rec.first_row = static_cast<int>(e.log_rows.size());
+    rec.n_rows = t.b;
+    e.log_tasks.push_back(rec);
+    for (const TaskRow& tr : t.rows) e.log_rows.push_back({e.reqs[tr.req].id, tr.node, tr.slot});
+  }
+  if (!e.device()) return BM_OK;
+  // ring placement: one contiguous region for all tasks of this Schedule call
+  if (total > e.ring_rows) return BM_E_INVAL;
+  if (e.ring_head + total > e.ring_rows) e.ring_head = 0;
+  const int base = e.ring_head;
+  int off = base;
+  for (Task& t : tasks) {
+    t.ring_off = off;
+    Cell& c = e.cells[t.ct];
+    for (int i = 0; i < t.b; ++i) e.ring_host[off + i] = make_row(e, c, t.rows[i]);
+    off += t.b;
+  }
+  e.ring_head = off;
+  CK(cudaMemcpyAsync(e.ring_dev + base, e.ring_host + base, sizeof(RowDesc) * total,
+                     cudaMemcpyHostToDevice, e.stream));
+  for (Task& t : tasks) {
+    bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, t.b, &t);
+    if (s != BM_OK) return s;
+    CK(launch_signal(e.signal_dev, e.stream));
+    e.stats.kernel_launches += 1;
+  }
+  return BM_OK;
+}
+
+// Retire every in-flight task the device has finished (and, on the virtual clock, whose tick
+// has come). Returns the number retired.
+static int retire_ready(Engine& e, bool block) {
+  int n = 0;
+  while (!e.inflight.empty()) {
+    Task& t = e.inflight.front();
+    if (e.cfg.clock != BM_CLOCK_WALL && t.finish > e.now) break;
+    if (e.device()) {
+      volatile unsigned long long* sig = e.signal_host;
+      if (*sig <= t.seq) {
+        if (!block && e.cfg.clock == BM_CLOCK_WALL) break;
+        while (*sig <= t.seq) {
+        }
+      }
+    }
+    if (e.cfg.clock == BM_CLOCK_WALL) e.now = wall_now(e);
+    retire_task(e, t);
+    if (t.ev_count > 0) {
+      for (int k = 0; k < t.ev_count; ++k) {
+        TimedLaunch& tl = e.ev_pool[(t.ev_first + k) % e.ev_pool.size()];
+        float ms = 0;
+        if (cudaEventElapsedTime(&ms, tl.beg, tl.end) == cudaSuccess) {
+          e.stats.timed_launches += 1;
+          e.stats.timed_ms += ms;
+          e.stats.timed_bytes += tl.bytes;
+          e.stats.timed_flops += tl.flops;
+        }
+      }
+    }
+    e.inflight.pop_front();
+    ++n;
+  }
+  return n;
+}
+
+static void admit_due(Engine& e) {
+  while (!e.pending.empty() && e.reqs[e.pending.front()].t_arrival <= e.now) {
+    const int ri = e.pending.front();
+    e.pending.pop_front();
+    admit_request(e, ri);
+  }
+}
+
+static bm_status schedule_and_launch(Engine& e, int* n_tasks) {
+  *n_tasks = 0;
+  if (static_cast<int>(e.inflight.size()) > e.cfg.schedule_when_outstanding_leq) return BM_OK;
+  static thread_local std::vector<Task> tasks;
+  tasks.clear();
+  const auto t0 = std::chrono::steady_clock::now();
+  schedule(e, tasks);
+  e.stats.sched_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
+  e.stats.schedule_calls += 1;
+  if (tasks.empty()) return BM_OK;
+  bm_status s = launch_tasks(e, tasks);
+  if (s != BM_OK) return s;
+  for (Task& t : tasks) e.inflight.push_back(std::move(t));
+  *n_tasks = static_cast<int>(tasks.size());
+  return BM_OK;
+}
+
+static bool all_done(const Engine& e) {
+  return e.pending.empty() && e.inflight.empty() && !has_ready(e);
+}
+
+// One round of the virtual-time event loop (S21); advances the clock to the next event.
+static bm_status virtual_round(Engine& e, int* n_tasks) {
+  retire_ready(e, true);
+  admit_due(e);
+  bm_status s = schedule_and_launch(e, n_tasks);
+  if (s != BM_OK) return s;
+  double next = 1e300;
+  if (!e.inflight.empty()) next = std::min(next, e.inflight.front().finish);
+  if (!e.pending.empty()) next = std::min(next, e.reqs[e.pending.front()].t_arrival);
+  if (next == 1e300) return all_done(e) ? BM_E_AGAIN : BM_E_STATE;  // nothing can progress
+  e.now = next;
+  return BM_OK;
+}
+
+}  // namespace bm
+
+using namespace bm;
+
+// ================================================================= C-ABI
+extern "C" {
+
+int bm_abi_version(void) { return BM_ABI_VERSION; }
+
+const char* bm_strerror(bm_status s) {
+  switch (s) {
+    case BM_OK: return "ok";
+    case BM_E_INVAL: return "invalid argument";
+    case BM_E_NOMEM: return "out of memory";
+    case BM_E_FULL: return "request table full";
+    case BM_E_AGAIN: return "nothing to do";
+    case BM_E_CUDA: return "CUDA error (sticky)";
+    case BM_E_STATE: return "invalid state";
+    case BM_E_NODEV: return "no sm_100 device";
+  }
+  return "unknown";
+}
+
+void bm_config_default(bm_config* c) {
+  memset(c, 0, sizeof(*c));
+  c->device = 0;
+  c->precision = BM_PREC_BF16;
+  c->clock = BM_CLOCK_WALL;
+  c->hidden = 1024;
+  c->pool_layers = 1;
+  c->max_slots = 65536;
+  c->max_requests = 65536;
+  c->max_tasks_to_submit = 5;
+  c->min_followon_batch = 1;
+  c->schedule_when_outstanding_leq = 0;
+  c->max_decode_len = 512;
+  c->keep_results = 0;
+  c->record_logits = 0;
+  c->time_kernels = 0;
+}
+
+static void free_device(Engine& e) {
+  if (!e.device()) return;
+  for (Cell& c : e.cells) {
+    for (void* p : c.W) cudaFree(p);
+    for (float* p : c.bias) cudaFree(p);
+    cudaFree(c.E);
+    cudaFree(c.W_out);
+    cudaFree(c.b_out);
+  }
+  cudaFree(e.h_pool);
+  cudaFree(e.c_pool);
+  cudaFree(e.tok);
+  cudaFree(e.res_h);
+  cudaFree(e.res_c);
+  cudaFree(e.res_tok);
+  cudaFree(e.logits);
+  cudaFree(e.amax);
+  cudaFree(e.done_ctas);
+  cudaFree(e.ring_dev);
+  cudaFree(e.direct_rows);
+  if (e.ring_host) cudaFreeHost(e.ring_host);
+  if (e.signal_host) cudaFreeHost(e.signal_host);
+  for (TimedLaunch& t : e.ev_pool) {
+    cudaEventDestroy(t.beg);
+    cudaEventDestroy(t.end);
+  }
+  if (e.stream) cudaStreamDestroy(e.stream);
+}
+
+bm_status bm_create(const bm_config* cfg, bm_engine** out) {
+  if (cfg == nullptr || out == nullptr) return BM_E_INVAL;
+  const bm_config& c = *cfg;
+  if (c.hidden <= 0 || c.hidden % 64 != 0 || c.pool_layers < 1 || c.pool_layers > 8 ||
+      c.max_slots < 1 || c.max_requests < 1 || c.max_requests >= (1 << 23) ||
+      c.max_tasks_to_submit < 1 || c.min_followon_batch < 1 || c.schedule_when_outstanding_leq < 0 ||
+      c.max_decode_len < 1 || c.precision < 0 || c.precision > 1 || c.clock < 0 || c.clock > 2)
+    return BM_E_INVAL;
+  Engine* e = new (std::nothrow) Engine();
+  if (e == nullptr) return BM_E_NOMEM;
+  e->cfg = c;
+  e->reqs.resize(c.max_requests);
+  e->free_slots_heap.resize(c.max_slots);
+  for (int i = 0; i < c.max_slots; ++i) e->free_slots_heap[i] = i;  // sorted == valid min-heap
+  e->t0 = std::chrono::steady_clock::now();
+  if (e->device()) {
+    Engine& E = *e;
+    auto fail = [&](bm_status s) {
+      free_device(E);
+      delete e;
+      return s;
+    };
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= c.device) return fail(BM_E_NODEV);
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, c.device) != cudaSuccess || prop.major != 10)
+      return fail(BM_E_NODEV);
+    if (cudaSetDevice(c.device) != cudaSuccess) return fail(BM_E_NODEV);
+    if (cudaStreamCreateWithFlags(&E.stream, cudaStreamNonBlocking) != cudaSuccess) return fail(BM_E_CUDA);
+    const size_t H = c.hidden, S = c.max_slots, L = c.pool_layers, R = c.max_requests;
+    const size_t el = E.elem();
+    bool ok = cudaMalloc(&E.h_pool, L * 2 * S * H * el) == cudaSuccess &&
+              dalloc(&E.c_pool, L * S * H) == cudaSuccess && dalloc(&E.tok, S) == cudaSuccess &&
+              dalloc(&E.res_h, R * L * H) == cudaSuccess && dalloc(&E.res_c, R * L * H) == cudaSuccess &&
+              dalloc(&E.res_tok, R * static_cast<size_t>(c.max_decode_len)) == cudaSuccess &&
+              dalloc(&E.amax, 512) == cudaSuccess && dalloc(&E.done_ctas, 1) == cudaSuccess &&
+              dalloc(&E.direct_rows, 4096) == cudaSuccess;
+    if (!ok) return fail(BM_E_NOMEM);
+    E.ring_rows = std::max(64, c.max_tasks_to_submit + c.schedule_when_outstanding_leq + 2) * 512 * 2;
+    if (dalloc(&E.ring_dev, E.ring_rows) != cudaSuccess) return fail(BM_E_NOMEM);
+    if (cudaHostAlloc(reinterpret_cast<void**>(&E.ring_host), E.ring_rows * sizeof(RowDesc),
+                      cudaHostAllocDefault) != cudaSuccess)
+      return fail(BM_E_NOMEM);
+    if (cudaHostAlloc(reinterpret_cast<void**>(&E.signal_host), sizeof(unsigned long long),
+                      cudaHostAllocMapped) != cudaSuccess)
+      return fail(BM_E_NOMEM);
+    *E.signal_host = 0;
+    if (cudaHostGetDevicePointer(reinterpret_cast<void**>(&E.signal_dev), E.signal_host, 0) != cudaSuccess)
+      return fail(BM_E_CUDA);
+    if (cudaMemsetAsync(E.h_pool, 0, L * 2 * S * H * el, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.c_pool, 0, L * S * H * 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.tok, 0, S * 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.amax, 0, 512 * 8, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.done_ctas, 0, 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.res_tok, 0, R * c.max_decode_len * 4, E.stream) != cudaSuccess)
+      return fail(BM_E_CUDA);
+    if (c.time_kernels) {
+      E.ev_pool.resize(4096);
+      for (TimedLaunch& t : E.ev_pool) {
+        if (cudaEventCreate(&t.beg) != cudaSuccess || cudaEventCreate(&t.end) != cudaSuccess)
+          return fail(BM_E_CUDA);
+      }
+    }
+    if (cudaStreamSynchronize(E.stream) != cudaSuccess) return fail(BM_E_CUDA);
+  }
+  *out = reinterpret_cast<bm_engine*>(e);
+  return BM_OK;
+}
+
+void bm_destroy(bm_engine* h) {
+  if (h == nullptr) return;
+  Engine* e = reinterpret_cast<Engine*>(h);
+  if (e->device() && e->stream) cudaStreamSynchronize(e->stream);
+  free_device(*e);
+  delete e;
+}
+
+void* bm_stream(bm_engine* h) { return h ? reinterpret_cast<Engine*>(h)->stream : nullptr; }
+
+bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w, int* cell_id) {
+  if (h == nullptr || d == nullptr || w == nullptr || cell_id == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  if (e.submitted_any) return BM_E_STATE;
+  if (e.cells.size() >= 64) return BM_E_INVAL;
+  const int H = e.cfg.hidden;
+  if (d->hidden != H || d->max_batch < 1 || d->max_batch > 512) return BM_E_INVAL;
+  Cell c;
+  c.d = *d;
+  switch (d->kind) {
+    case BM_CELL_LSTM:
+    case BM_CELL_LSTM_PROJ:
+      if (d->layers < 1 || d->layers > e.cfg.pool_layers || d->vocab < 1) return BM_E_INVAL;
+      if (d->kind == BM_CELL_LSTM_PROJ && (d->vocab % 128 != 0 || w->W_out == nullptr || w->b_out == nullptr))
+        return BM_E_INVAL;
+      c.epi = EPI_LSTM, c.G = 4, c.U = 32, c.K0 = H, c.K1 = H;
+      break;
+    case BM_CELL_TREE_LEAF:
+      if (d->layers != 1 || d->vocab < 1) return BM_E_INVAL;
+      c.epi = EPI_LEAF, c.G = 3, c.U = 32, c.K0 = H, c.K1 = 0;
+      break;
+    case BM_CELL_TREE_INTERNAL:
+      if (d->layers != 1) return BM_E_INVAL;
+      c.epi = EPI_INTERNAL, c.G = 5, c.U = 16, c.K0 = H, c.K1 = H;
+      break;
+    default:
+      return BM_E_INVAL;
+  }
+  const int K = c.K0 + c.K1;
+  c.S = std::max(1, K / 512);          // fixed K slice of 512 -> batch-invariant reduction order
+  c.kslice = K / c.S;
+  if (c.S > 8 || c.kslice % 64 != 0) return BM_E_INVAL;
+  if (w->W == nullptr || w->b == nullptr) return BM_E_INVAL;
+  const int L = (d->kind == BM_CELL_LSTM || d->kind == BM_CELL_LSTM_PROJ) ? d->layers : 1;
+  for (int l = 0; l < L; ++l)
+    if (w->W[l] == nullptr || w->b[l] == nullptr) return BM_E_INVAL;
+  if (d->kind != BM_CELL_TREE_INTERNAL && w->E == nullptr) return BM_E_INVAL;
+  if (e.device()) {
+    const bool bf = e.cfg.precision == BM_PREC_BF16;
+    const size_t el = e.elem();
+    const size_t rows = static_cast<size_t>(c.G) * H;
+    float* tmp = nullptr;
+    float* tmpb = nullptr;
+    const size_t maxsrc = std::max(rows * K, static_cast<size_t>(d->vocab) * H);
+    CK(cudaMalloc(&tmp, maxsrc * 4));
+    CK(cudaMalloc(&tmpb, std::max(rows, static_cast<size_t>(d->vocab)) * 4));
+    for (int l = 0; l < L; ++l) {
+      void* Wp = nullptr;
+      float* bp = nullptr;
+      CK(cudaMalloc(&Wp, rows * K * el));
+      CK(dalloc(&bp, rows));
+      CK(cudaMemcpyAsync(tmp, w->W[l], rows * K * 4, cudaMemcpyHostToDevice, e.stream));
+      CK(cudaMemcpyAsync(tmpb, w->b[l], rows * 4, cudaMemcpyHostToDevice, e.stream));
+      CK(launch_pack_rows(tmp, Wp, bp, tmpb, c.G, H, K, bf ? 1 : 0, e.stream));
+      CK(cudaStreamSynchronize(e.stream));
+      c.W.push_back(Wp);
+      c.bias.push_back(bp);
+      if (bf) {
+        CUtensorMap m;
+        if (!make_tmap(&m, Wp, static_cast<int>(rows), K, c.G * c.U)) return BM_E_CUDA;
+        c.tm.push_back(m);
+      }
+    }
+    if (w->E != nullptr && d->kind != BM_CELL_TREE_INTERNAL) {
+      const size_t n = static_cast<size_t>(d->vocab) * H;
+      CK(cudaMalloc(&c.E, n * el));
+      CK(cudaMemcpyAsync(tmp, w->E, n * 4, cudaMemcpyHostToDevice, e.stream));
+      CK(launch_convert(tmp, c.E, n, bf ? 1 : 0, e.stream));
+      CK(cudaStreamSynchronize(e.stream));
+    }
+    if (d->kind == BM_CELL_LSTM_PROJ) {
+      const size_t n = static_cast<size_t>(d->vocab) * H;
+      CK(cudaMalloc(&c.W_out, n * el));
+      CK(dalloc(&c.b_out, d->vocab));
+      CK(cudaMemcpyAsync(tmp, w->W_out, n * 4, cudaMemcpyHostToDevice, e.stream));
+      CK(launch_convert(tmp, c.W_out, n, bf ? 1 : 0, e.stream));
+      CK(cudaMemcpyAsync(c.b_out, w->b_out, d->vocab * 4, cudaMemcpyHostToDevice, e.stream));
+      CK(cudaStreamSynchronize(e.stream));
+      if (bf && !make_tmap(&c.tm_out, c.W_out, d->vocab, H, 128)) return BM_E_CUDA;
+      if (e.cfg.record_logits) {
+        if (e.logits == nullptr) {
+          CK(dalloc(&e.logits, static_cast<size_t>(e.cfg.max_requests) * e.cfg.max_decode_len * d->vocab));
+          e.logits_vocab = d->vocab;
+        } else if (e.logits_vocab != d->vocab) {
+          return BM_E_INVAL;
+        }
+      }
+    }
+    cudaFree(tmp);
+    cudaFree(tmpb);
+  }
+  e.cells.push_back(c);
+  *cell_id = static_cast<int>(e.cells.size()) - 1;
+  return BM_OK;
+}
+
+static bool valid_tree(const bm_request* r) {
+  const int n = r->n;
+  if (n < 1 || r->left == nullptr || r->right == nullptr) return false;
+  std::vector<int> parents(n, 0);
+  for (int v = 0; v < n; ++v) {
+    const int L = r->left[v], R = r->right[v];
+    if ((L < 0) != (R < 0)) return false;       // binary: both children or none
+    if (L >= 0) {
+      if (L >= v || R >= v || L == R) return false;   // post-order: children first
+      parents[L]++;
+      parents[R]++;
+    }
+  }
+  for (int v = 0; v < n - 1; ++v)
+    if (parents[v] != 1) return false;
+  return parents[n - 1] == 0;
+}
+
+bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
+  if (h == nullptr || q == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  const int nc = static_cast<int>(e.cells.size());
+  auto cell_ok = [&](int id, int k1, int k2) {
+    return id >= 0 && id < nc && (e.cells[id].d.kind == k1 || e.cells[id].d.kind == k2);
+  };
+  if (q->n < 1 || q->tokens == nullptr) return BM_E_INVAL;
+  int vocab = 0;
+  if (q->kind == BM_REQ_CHAIN) {
+    if (!cell_ok(q->cell0, BM_CELL_LSTM, BM_CELL_LSTM)) return BM_E_INVAL;
+    vocab = e.cells[q->cell0].d.vocab;
+  } else if (q->kind == BM_REQ_SEQ2SEQ) {
+    if (!cell_ok(q->cell0, BM_CELL_LSTM, BM_CELL_LSTM) || !cell_ok(q->cell1, BM_CELL_LSTM_PROJ, BM_CELL_LSTM_PROJ))
+      return BM_E_INVAL;
+    if (q->decode_len < 1 || q->decode_len > e.cfg.max_decode_len) return BM_E_INVAL;
+    if (e.cells[q->cell0].d.layers != e.cells[q->cell1].d.layers) return BM_E_INVAL;
+    vocab = e.cells[q->cell0].d.vocab;
+  } else if (q->kind == BM_REQ_TREE) {
+    if (!cell_ok(q->cell0, BM_CELL_TREE_LEAF, BM_CELL_TREE_LEAF) ||
+        !cell_ok(q->cell1, BM_CELL_TREE_INTERNAL, BM_CELL_TREE_INTERNAL) || !valid_tree(q))
+      return BM_E_INVAL;
+    if (q->n > e.cfg.max_slots) return BM_E_INVAL;
+    vocab = e.cells[q->cell0].d.vocab;
+  } else {
+    return BM_E_INVAL;
+  }
+  for (int i = 0; i < q->n; ++i) {
+    const bool leaf_or_chain = q->kind != BM_REQ_TREE || q->left[i] < 0;
+    if (leaf_or_chain && (q->tokens[i] < 0 || q->tokens[i] >= vocab)) return BM_E_INVAL;
+  }
+  if (e.n_live_reqs >= e.cfg.max_requests) return BM_E_FULL;
+  // request table slot: the entry of admission index id % max_requests must be free
+  const int ri = static_cast<int>(e.next_req_id % e.cfg.max_requests);
+  Request& r = e.reqs[ri];
+  if (r.used) return BM_E_FULL;
+  r.used = true;
+  r.done = false;
+  r.id = e.next_req_id++;
+  r.tag = q->user_tag;
+  r.kind = q->kind;
+  r.cell0 = q->cell0;
+  r.cell1 = q->cell1;
+  r.t_arrival = q->arrival;
+  r.tokens.assign(q->tokens, q->tokens + q->n);
+  if (q->kind == BM_REQ_CHAIN) {
+    r.n_nodes = q->n;
+    r.enc_len = q->n;
+  } else if (q->kind == BM_REQ_SEQ2SEQ) {
+    r.enc_len = q->n;
+    r.n_nodes = q->n + q->decode_len;
+  } else {
+    r.n_nodes = q->n;
+    r.left.assign(q->left, q->left + q->n);
+    r.right.assign(q->right, q->right + q->n);
+  }
+  e.n_live_reqs += 1;
+  e.submitted_any = true;
+  e.pending.push_back(ri);
+  if (req_id) *req_id = r.id;
+  return BM_OK;
+}
+
+bm_status bm_schedule_step(bm_engine* h, int* n_tasks) {
+  if (h == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  int n = 0;
+  bm_status s;
+  if (e.cfg.clock == BM_CLOCK_WALL) {
+    if (!e.wall_started) {
+      e.t0 = std::chrono::steady_clock::now();
+      e.wall_started = true;
+    }
+    e.now = wall_now(e);
+    retire_ready(e, false);
+    admit_due(e);
+    s = schedule_and_launch(e, &n);
+    if (s == BM_OK && n == 0 && all_done(e)) s = BM_E_AGAIN;
+  } else {
+    s = virtual_round(e, &n);
+  }
+  if (n_tasks) *n_tasks = n;
+  return s;
+}
+
+bm_status bm_poll(bm_engine* h, bm_completion* out, int cap, int* n) {
+  if (h == nullptr || n == nullptr || (cap > 0 && out == nullptr)) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.cfg.clock == BM_CLOCK_WALL) {
+    e.now = wall_now(e);
+    retire_ready(e, false);
+  }
+  const int k = std::min<int>(cap, static_cast<int>(e.completions.size()));
+  if (k > 0) memcpy(out, e.completions.data(), k * sizeof(bm_completion));
+  e.completions.erase(e.completions.begin(), e.completions.begin() + k);
+  *n = k;
+  return BM_OK;
+}
+
+bm_status bm_run(bm_engine* h, int* n_completed) {
+  if (h == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  const size_t before = e.completions.size();
+  int n = 0;
+  bm_status s = BM_OK;
+  if (e.cfg.clock == BM_CLOCK_WALL) {
+    e.t0 = std::chrono::steady_clock::now();
+    e.wall_started = true;
+    while (true) {
+      e.now = wall_now(e);
+      retire_ready(e, false);
+      admit_due(e);
+      s = schedule_and_launch(e, &n);
+      if (s != BM_OK) return s;
+      if (all_done(e)) break;
+    }
+  } else {
+    while ((s = virtual_round(e, &n)) == BM_OK) {
+    }
+    if (s != BM_E_AGAIN) return s;
+  }
+  if (e.device()) CK(cudaStreamSynchronize(e.stream));
+  if (n_completed) *n_completed = static_cast<int>(e.completions.size() - before);
+  return BM_OK;
+}
+
+bm_status bm_read_result(bm_engine* h, uint64_t req_id, bm_result* dst) {
+  if (h == nullptr || dst == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  Request& r = e.reqs[req_id % e.cfg.max_requests];
+  if (!r.used || r.id != req_id) return BM_E_INVAL;
+  if (!r.done) return BM_E_STATE;
+  if (!e.device()) return BM_E_STATE;
+  const int ri = static_cast<int>(req_id % e.cfg.max_requests);
+  const size_t H = e.H(), L = e.cfg.pool_layers;
+  CK(cudaStreamSynchronize(e.stream));
+  if (dst->h) CK(cudaMemcpy(dst->h, e.res_h + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost));
+  if (dst->c) CK(cudaMemcpy(dst->c, e.res_c + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost));
+  if (r.kind == BM_REQ_SEQ2SEQ) {
+    const int T = r.n_nodes - r.enc_len;
+    if (dst->tokens)
+      CK(cudaMemcpy(dst->tokens, e.res_tok + static_cast<size_t>(ri) * e.cfg.max_decode_len, T * 4,
+                    cudaMemcpyDeviceToHost));
+    if (dst->logits && e.logits)
+      CK(cudaMemcpy(dst->logits, e.logits + static_cast<size_t>(ri) * e.cfg.max_decode_len * e.logits_vocab,
+                    static_cast<size_t>(T) * e.logits_vocab * 4, cudaMemcpyDeviceToHost));
+  }
+  return BM_OK;
+}
+
+bm_status bm_release(bm_engine* h, uint64_t req_id) {
+  if (h == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  Request& r = e.reqs[req_id % e.cfg.max_requests];
+  if (!r.used || r.id != req_id) return BM_E_INVAL;
+  if (!r.done) return BM_E_STATE;
+  r.used = false;
+  e.n_live_reqs -= 1;
+  return BM_OK;
+}
+
+bm_status bm_read_log(bm_engine* h, bm_task_record* out, int cap, int* n) {
+  if (h == nullptr || n == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  const int k = std::min<int>(cap, static_cast<int>(e.log_tasks.size()));
+  if (k > 0) memcpy(out, e.log_tasks.data(), k * sizeof(bm_task_record));
+  *n = static_cast<int>(e.log_tasks.size());
+  return BM_OK;
+}
+
+bm_status bm_read_log_rows(bm_engine* h, bm_row_record* out, int cap, int* n) {
+  if (h == nullptr || n == nullptr) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  const int k = std::min<int>(cap, static_cast<int>(e.log_rows.size()));
+  if (k > 0) memcpy(out, e.log_rows.data(), k * sizeof(bm_row_record));
+  *n = static_cast<int>(e.log_rows.size());
+  return BM_OK;
+}
+
+bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b, int async) {
+  if (h == nullptr || rows == nullptr || b < 1 || b > 4096) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  if (!e.device()) return BM_E_STATE;
+  if (cell_id < 0 || cell_id >= static_cast<int>(e.cells.size())) return BM_E_INVAL;
+  Cell& c = e.cells[cell_id];
+  if (c.d.kind == BM_CELL_LSTM_PROJ && b > 512) return BM_E_INVAL;
+  for (int i = 0; i < b; ++i) {
+    if (rows[i].slot < 0 || rows[i].slot >= e.cfg.max_slots) return BM_E_INVAL;
+    if ((rows[i].flags >> 8) >= e.cfg.max_requests) return BM_E_INVAL;
+  }
+  CK(cudaMemcpyAsync(e.direct_rows, rows, sizeof(RowDesc) * b, cudaMemcpyHostToDevice, e.stream));
+  bm_status s = launch_cell(e, c, e.direct_rows, b, nullptr);
+  if (s != BM_OK) return s;
+  if (!async) CK(cudaStreamSynchronize(e.stream));
+  return BM_OK;
+}
+
+static bm_status pool_io(Engine& e, int layer, int parity, const int32_t* slots, int n, float* h,
+                         float* c, int write) {
+  if (!e.device()) return BM_E_STATE;
+  if (layer < 0 || layer >= e.cfg.pool_layers || parity < 0 || parity > 1 || n < 1 || slots == nullptr)
+    return BM_E_INVAL;
+  for (int i = 0; i < n; ++i)
+    if (slots[i] < 0 || slots[i] >= e.cfg.max_slots) return BM_E_INVAL;
+  const size_t H = e.H();
+  int32_t* ds = nullptr;
+  float *dh = nullptr, *dc = nullptr;
+  CK(cudaMalloc(&ds, n * 4));
+  CK(cudaMalloc(&dh, n * H * 4));
+  CK(cudaMalloc(&dc, n * H * 4));
+  CK(cudaMemcpy(ds, slots, n * 4, cudaMemcpyHostToDevice));
+  if (write) {
+    if (h) CK(cudaMemcpy(dh, h, n * H * 4, cudaMemcpyHostToDevice));
+    if (c) CK(cudaMemcpy(dc, c, n * H * 4, cudaMemcpyHostToDevice));
+  }
+  void* hp = static_cast<char*>(e.h_layer(layer)) + static_cast<size_t>(parity) * e.cfg.max_slots * H * e.elem();
+  CK(launch_pool_io(hp, e.c_layer(layer), ds, n, static_cast<int>(H), h ? dh : nullptr,
+                    c ? dc : nullptr, write, e.cfg.precision == BM_PREC_BF16, e.stream));
+  CK(cudaStreamSynchronize(e.stream));
+  if (!write) {
+    if (h) CK(cudaMemcpy(h, dh, n * H * 4, cudaMemcpyDeviceToHost));
+    if (c) CK(cudaMemcpy(c, dc, n * H * 4, cudaMemcpyDeviceToHost));
+  }
+  cudaFree(ds);
+  cudaFree(dh);
+  cudaFree(dc);
+  return BM_OK;
+}
+
+bm_status bm_pool_write(bm_engine* h, int layer, int parity, const int32_t* slots, int n,
+                        const float* hh, const float* cc) {
+  if (h == nullptr) return BM_E_INVAL;
+  return pool_io(*reinterpret_cast<Engine*>(h), layer, parity, slots, n, const_cast<float*>(hh),
+                 const_cast<float*>(cc), 1);
+}
+
+bm_status bm_pool_read(bm_engine* h, int layer, int parity, const int32_t* slots, int n, float* hh,
+                       float* cc) {
+  if (h == nullptr) return BM_E_INVAL;
+  return pool_io(*reinterpret_cast<Engine*>(h), layer, parity, slots, n, hh, cc, 0);
+}
+
+bm_status bm_result_rows(bm_engine* h, const int32_t* res_idx, int n, float* hh, float* cc) {
+  if (h == nullptr || res_idx == nullptr || n < 1) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (!e.device()) return BM_E_STATE;
+  const size_t LH = e.H() * e.cfg.pool_layers;
+  CK(cudaStreamSynchronize(e.stream));
+  for (int i = 0; i < n; ++i) {
+    if (res_idx[i] < 0 || res_idx[i] >= e.cfg.max_requests) return BM_E_INVAL;
+    if (hh) CK(cudaMemcpy(hh + i * LH, e.res_h + res_idx[i] * LH, LH * 4, cudaMemcpyDeviceToHost));
+    if (cc) CK(cudaMemcpy(cc + i * LH, e.res_c + res_idx[i] * LH, LH * 4, cudaMemcpyDeviceToHost));
+  }
+  return BM_OK;
+}
+
+bm_status bm_tokens(bm_engine* h, const int32_t* slots, int n, int32_t* inout, int write) {
+  if (h == nullptr || slots == nullptr || inout == nullptr || n < 1) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (!e.device()) return BM_E_STATE;
+  CK(cudaStreamSynchronize(e.stream));
+  for (int i = 0; i < n; ++i) {
+    if (slots[i] < 0 || slots[i] >= e.cfg.max_slots) return BM_E_INVAL;
+    if (write) CK(cudaMemcpy(e.tok + slots[i], inout + i, 4, cudaMemcpyHostToDevice));
+    else CK(cudaMemcpy(inout + i, e.tok + slots[i], 4, cudaMemcpyDeviceToHost));
+  }
+  return BM_OK;
+}
+
+bm_status bm_get_stats(bm_engine* h, bm_stats* out) {
+  if (h == nullptr || out == nullptr) return BM_E_INVAL;
+  *out = reinterpret_cast<Engine*>(h)->stats;
+  return BM_OK;
+}
+
+bm_status bm_reset_stats(bm_engine* h) {
+  if (h == nullptr) return BM_E_INVAL;
+  reinterpret_cast<Engine*>(h)->stats = bm_stats{};
+  return BM_OK;
+}
+
+}  // extern "C"

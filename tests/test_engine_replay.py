@@ -1,0 +1,154 @@
+"""P9 on CPU: the C++ engine's scheduler (libbm.so, BM_CLOCK_DRY: no device work) produces
+exactly the task log, slot indices and completion order/ticks of the independent Python replay
+of Algorithm 1 (oracle/scheduler.py) for the same arrival trace."""
+import numpy as np
+import pytest
+from hypothesis import HealthCheck, given, settings
+from hypothesis import strategies as st
+
+from oracle.scheduler import CHAIN, SEQ2SEQ, TREE, Replay
+from paper_conf_eurosys_gaoywl18_b200 import bm
+from workloads import gen
+
+H = 64
+V = 16
+
+
+def _engine(cts, clock=bm.CLOCK_DRY, **kw):
+    """cts: list of (kind, bmax, priority). Weights are zeros (DRY: never used)."""
+    e = bm.Engine(clock=clock, hidden=H, pool_layers=2, **kw)
+    ids = []
+    for kind, bmax, prio in cts:
+        if kind == bm.CELL_TREE_LEAF:
+            W, b, E = [np.zeros((3 * H, H), np.float32)], [np.zeros(3 * H, np.float32)], np.zeros((V, H), np.float32)
+            ids.append(e.load_cell(kind, 1, V, bmax, prio, W, b, E))
+        elif kind == bm.CELL_TREE_INTERNAL:
+            ids.append(e.load_cell(kind, 1, V, bmax, prio, [np.zeros((5 * H, 2 * H), np.float32)],
+                                   [np.zeros(5 * H, np.float32)]))
+        else:
+            W = [np.zeros((4 * H, 2 * H), np.float32)] * 2
+            b = [np.zeros(4 * H, np.float32)] * 2
+            kw2 = {}
+            if kind == bm.CELL_LSTM_PROJ:
+                kw2 = dict(W_out=np.zeros((128, H), np.float32), b_out=np.zeros(128, np.float32))
+            ids.append(e.load_cell(kind, 2, 128 if kind == bm.CELL_LSTM_PROJ else V, bmax, prio, W, b,
+                                   np.zeros((128 if kind == bm.CELL_LSTM_PROJ else V, H), np.float32), **kw2))
+    return e, ids
+
+
+def _submit_all(e, reqs):
+    for q in reqs:
+        if q["kind"] == CHAIN:
+            e.submit(bm.REQ_CHAIN, q["cells"][0], 0, [3] * q["length"], q["arrival"])
+        elif q["kind"] == SEQ2SEQ:
+            e.submit(bm.REQ_SEQ2SEQ, q["cells"][0], q["cells"][1], [3] * q["length"], q["arrival"],
+                     decode_len=q["decode_len"])
+        else:
+            n = len(q["left"])
+            e.submit(bm.REQ_TREE, q["cells"][0], q["cells"][1], [3] * n, q["arrival"],
+                     left=q["left"], right=q["right"])
+
+
+def _compare(e, rp):
+    log = e.read_log()
+    assert len(log) == len(rp.tasks)
+    for a, t in zip(log, rp.tasks):
+        assert a["cell"] == t.ct
+        assert a["tick"] == t.tick
+        assert a["rows"] == [(r.rid, r.node, r.slot) for r in t.rows]
+    comp = e.poll()
+    assert [(c.req_id, c.t_done) for c in comp] == [(rid, float(tk)) for rid, tk in rp.completions]
+    for c in comp:
+        r = rp.reqs[c.req_id]
+        assert c.t_first == r.first_tick
+
+
+def _chain_case(trace, bmax, minf, max_tasks=5, k=0, slots=1 << 12):
+    e, ids = _engine([(bm.CELL_LSTM, bmax, 0)], max_slots=slots, max_requests=1 << 12,
+                     min_followon_batch=minf, max_tasks_to_submit=max_tasks,
+                     schedule_when_outstanding_leq=k)
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": q.arrival, "length": q.length} for q in trace]
+    _submit_all(e, reqs)
+    e.run()
+    rp = Replay([(bmax, 0)], max_slots=slots, max_tasks_to_submit=max_tasks, min_followon=minf,
+                schedule_when_outstanding_leq=k).run(reqs)
+    _compare(e, rp)
+
+
+@pytest.mark.parametrize("minf", [1, 4])
+def test_figure5_replay(minf):
+    _chain_case(gen.figure5_trace(), 4, minf)
+
+
+@pytest.mark.parametrize("minf", [1, 4])
+def test_config0_replay(minf):
+    _chain_case(gen.config0_trace(), 4, minf)
+
+
+def test_wmt_poisson_replay():
+    trace = gen.chain_trace(400, 64, 7, rate=3.0)
+    _chain_case(trace, 32, 1, k=2, slots=64)
+
+
+def test_complete_tree_replay():
+    left, right = gen.complete_tree(16)
+    reqs = [{"kind": TREE, "cells": [0, 1], "arrival": 0, "left": left, "right": right}]
+    e, _ = _engine([(bm.CELL_TREE_LEAF, 64, 0), (bm.CELL_TREE_INTERNAL, 64, 1)], max_slots=256,
+                   max_requests=16)
+    _submit_all(e, reqs)
+    e.run()
+    _compare(e, Replay([(64, 0), (64, 1)], max_slots=256).run(reqs))
+
+
+def _random_reqs(seed, n, kinds):
+    rng = np.random.default_rng(seed)
+    out = []
+    t = 0.0
+    for _ in range(n):
+        t += float(rng.integers(0, 3))
+        kind = kinds[int(rng.integers(0, len(kinds)))]
+        if kind == CHAIN:
+            out.append({"kind": CHAIN, "cells": [0], "arrival": t, "length": int(rng.integers(1, 9))})
+        elif kind == SEQ2SEQ:
+            out.append({"kind": SEQ2SEQ, "cells": [1, 2], "arrival": t,
+                        "length": int(rng.integers(1, 6)), "decode_len": int(rng.integers(1, 6))})
+        else:
+            left, right = gen._random_bracketing(int(rng.integers(1, 9)), rng)
+            out.append({"kind": TREE, "cells": [3, 4], "arrival": t, "left": left, "right": right})
+    return out
+
+
+@settings(max_examples=200, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 100_000), n=st.integers(1, 20),
+       bmax=st.lists(st.integers(1, 6), min_size=5, max_size=5),
+       prio=st.permutations([0, 1, 2, 3, 4]), max_tasks=st.integers(1, 5),
+       min_followon=st.integers(1, 4), k=st.integers(0, 3), slots=st.integers(4, 40),
+       kinds=st.sampled_from([[CHAIN], [SEQ2SEQ], [TREE], [CHAIN, SEQ2SEQ, TREE]]))
+def test_random_traces_bit_exact(seed, n, bmax, prio, max_tasks, min_followon, k, slots, kinds):
+    reqs = _random_reqs(seed, n, kinds)
+    need = max((len(q["left"]) if q["kind"] == TREE else 1) for q in reqs)
+    slots = max(slots, need)
+    kinds_c = [bm.CELL_LSTM, bm.CELL_LSTM, bm.CELL_LSTM_PROJ, bm.CELL_TREE_LEAF, bm.CELL_TREE_INTERNAL]
+    e, _ = _engine(list(zip(kinds_c, bmax, prio)), max_slots=slots, max_requests=64,
+                   max_tasks_to_submit=max_tasks, min_followon_batch=min_followon,
+                   schedule_when_outstanding_leq=k)
+    _submit_all(e, reqs)
+    e.run()
+    rp = Replay(list(zip(bmax, prio)), max_slots=slots, max_tasks_to_submit=max_tasks,
+                min_followon=min_followon, schedule_when_outstanding_leq=k).run(reqs)
+    _compare(e, rp)
+
+
+def test_schedule_step_api_matches_run():
+    """Driving the engine with bm_schedule_step (the paper's per-idle Schedule call) gives the
+    same log as bm_run."""
+    trace = gen.config0_trace()
+    e, _ = _engine([(bm.CELL_LSTM, 4, 0)], max_slots=16, max_requests=16)
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": q.arrival, "length": q.length} for q in trace]
+    _submit_all(e, reqs)
+    n = 0
+    while e.schedule_step() >= 0:
+        n += 1
+        assert n < 1000
+    rp = Replay([(4, 0)], max_slots=16).run(reqs)
+    _compare(e, rp)

@@ -1,0 +1,141 @@
+"""End-to-end parity on the GPU (-m gpu): whole traces through the C-ABI engine (scheduler +
+kernels), checked two ways (north_star):
+  1. the scheduler's task log (batch composition, slot indices) and per-request completion
+     order are bit-exact with the Python replay of Algorithm 1 (virtual clock, P9);
+  2. every request's final h/c (and Seq2Seq tokens/logits) agree with the fp64 oracle run
+     unbatched, within 5e-3 (bf16) / 1e-5 (fp32)."""
+import numpy as np
+import pytest
+
+from oracle import cells
+from oracle.scheduler import CHAIN, SEQ2SEQ, TREE, Replay
+from paper_conf_eurosys_gaoywl18_b200 import bm
+from gpu_helpers import TOL, lstm_engine, seq2seq_engine, tree_engine
+from workloads import gen
+
+pytestmark = pytest.mark.gpu
+
+
+def _check_log(e, rp):
+    log = e.read_log()
+    assert len(log) == len(rp.tasks)
+    for a, t in zip(log, rp.tasks):
+        assert a["cell"] == t.ct and a["tick"] == t.tick
+        assert a["rows"] == [(r.rid, r.node, r.slot) for r in t.rows]
+    comp = e.poll()
+    assert [(c.req_id, c.t_done) for c in comp] == [(rid, float(tk)) for rid, tk in rp.completions]
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+@pytest.mark.parametrize("minf", [1, 4])
+def test_config0_end_to_end(prec, minf):
+    """BASELINE configs[0]: 1-layer LSTM, h=64, 4 requests (3, 10, 5, 8), arrivals (0, 0, 1, 3),
+    bmax 4, virtual clock."""
+    trace = gen.config0_trace(vocab=128)
+    e, cid, w = lstm_engine(64, 1, 128, prec, bmax=4, clock=bm.CLOCK_VIRTUAL, max_slots=16,
+                            max_requests=16, keep_results=1, min_followon_batch=minf)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    e.run()
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": q.arrival, "length": q.length} for q in trace]
+    _check_log(e, Replay([(4, 0)], max_slots=16, min_followon=minf).run(reqs))
+    for i, q in enumerate(trace):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, q.tokens)
+        assert np.max(np.abs(r["h"][0] - hs[0])) <= TOL[prec]
+        assert np.max(np.abs(r["c"][0] - cs[0])) <= TOL[prec]
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+def test_wmt_chain_h1024(prec):
+    """configs[1] shape at a size the oracle finishes in seconds: 48 WMT-length requests,
+    Poisson arrivals, h=1024, bmax 512, virtual clock with look-ahead k=2."""
+    trace = gen.chain_trace(48, 2048, seed=1000, rate=2.0)
+    e, cid, w = lstm_engine(1024, 1, 2048, prec, bmax=512, clock=bm.CLOCK_VIRTUAL, max_slots=256,
+                            max_requests=256, keep_results=1, schedule_when_outstanding_leq=2)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    e.run()
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": q.arrival, "length": q.length} for q in trace]
+    _check_log(e, Replay([(512, 0)], max_slots=256, schedule_when_outstanding_leq=2).run(reqs))
+    worst = 0.0
+    for i, q in enumerate(trace):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, q.tokens)
+        worst = max(worst, np.max(np.abs(r["h"][0] - hs[0])), np.max(np.abs(r["c"][0] - cs[0])))
+    assert worst <= TOL[prec], worst
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+@pytest.mark.parametrize("h,V,n", [(64, 256, 12), (1024, 32768, 6)])
+def test_seq2seq_forced_tokens(prec, h, V, n):
+    """Seq2Seq 4+4 layers, greedy feed-previous decoding on device. The oracle follows the GPU's
+    emitted tokens (forced-token mode) and asserts each was a valid argmax within tolerance;
+    then final h/c per layer and every step's logits are compared."""
+    L = 4
+    rng = np.random.default_rng(h)
+    e, (ce, cd), (enc, dec) = seq2seq_engine(h, L, V, prec, bmax=(512, 256), clock=bm.CLOCK_VIRTUAL,
+                                             max_slots=64, max_requests=64, keep_results=1,
+                                             record_logits=1, max_decode_len=40)
+    trace = []
+    for i in range(n):
+        S = int(rng.integers(1, 12))
+        T = int(rng.integers(1, 12))
+        trace.append((rng.integers(3, V, size=S).astype(np.int32), T, float(rng.integers(0, 6))))
+    trace.sort(key=lambda x: x[2])
+    for toks, T, t in trace:
+        e.submit(bm.REQ_SEQ2SEQ, ce, cd, toks, t, decode_len=T)
+    e.run()
+    reqs = [{"kind": SEQ2SEQ, "cells": [0, 1], "arrival": t, "length": len(toks), "decode_len": T}
+            for toks, T, t in trace]
+    _check_log(e, Replay([(512, 0), (256, 1)], max_slots=64).run(reqs))
+    tol = TOL[prec]
+    for i, (toks, T, _) in enumerate(trace):
+        r = e.read_result(i, L, decode_len=T, vocab=V)
+        o = cells.seq2seq(enc, dec, toks, T, forced_tokens=r["tokens"])
+        for s in range(T):
+            assert o["logits"][s][r["tokens"][s]] >= o["logits"][s].max() - 2 * tol
+        assert np.max(np.abs(r["logits"] - o["logits"])) <= tol
+        for l in range(L):
+            assert np.max(np.abs(r["h"][l] - o["h"][l])) <= tol
+            assert np.max(np.abs(r["c"][l] - o["c"][l])) <= tol
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+def test_treebank_trees_h1024(prec):
+    """configs[3] shape: TreeBank-like binary trees + the identical complete 16-leaf tree,
+    leaf and internal cell types batched separately (bmax 64), virtual clock."""
+    V = 4096
+    trace = gen.tree_trace(10, V, seed=3000, rate=1.0) + gen.tree_trace(2, V, seed=3001, identical=True)
+    for j, q in enumerate(trace):
+        q.arrival = float(j // 3)
+    e, (leaf, intern), w = tree_engine(1024, V, prec, bmax=64, clock=bm.CLOCK_VIRTUAL, max_slots=1024,
+                                       max_requests=64, keep_results=1)
+    for q in trace:
+        e.submit(bm.REQ_TREE, leaf, intern, q.tokens, q.arrival, left=q.left, right=q.right)
+    e.run()
+    reqs = [{"kind": TREE, "cells": [0, 1], "arrival": q.arrival, "left": q.left, "right": q.right}
+            for q in trace]
+    _check_log(e, Replay([(64, 0), (64, 1)], max_slots=1024).run(reqs))
+    for i, q in enumerate(trace):
+        r = e.read_result(i, 1)
+        rh, rc, _ = cells.tree_lstm(w, q.tokens, q.left, q.right)
+        assert np.max(np.abs(r["h"][0] - rh)) <= TOL[prec]
+        assert np.max(np.abs(r["c"][0] - rc)) <= TOL[prec]
+
+
+def test_wall_clock_run_completes_and_matches_oracle():
+    """The open-loop driver on the wall clock (bench path): all requests complete, results
+    match the oracle (scheduling then depends on timing, results must not)."""
+    trace = gen.chain_trace(64, 1024, seed=5, rate=20000.0)
+    e, cid, w = lstm_engine(1024, 1, 1024, bm.PREC_BF16, bmax=512, max_slots=256, max_requests=256,
+                            keep_results=1, schedule_when_outstanding_leq=2)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    assert e.run() == 64
+    comp = e.poll()
+    assert sorted(c.req_id for c in comp) == list(range(64))
+    for i in (0, 17, 63):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, trace[i].tokens)
+        assert np.max(np.abs(r["h"][0] - hs[0])) <= TOL[bm.PREC_BF16]
