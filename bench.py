@@ -1,0 +1,425 @@
+#!/usr/bin/env python
+"""bench.py -- requests/sec at a p90-latency bound for cellular batching on B200.
+
+Workload (BASELINE.json configs[1], the metric's configuration): 1-layer LSTM, h = 1024,
+WMT-like sentence lengths (mean 24, max 330; L421, L635), Poisson open-loop arrivals (L423),
+bmax 512 (L429), MaxTasksToSubmit 5 (L379), synthetic seeded weights/tokens.
+`--workload seq2seq|tree` runs configs[2] / configs[3] instead.
+
+A STEP = one open-loop Poisson trace of --reqs requests at the offered rate lambda* pushed
+through the whole hot path (A1 unfold at admission, A2-A3 Algorithm 1, A4 slot pool, A5 launch,
+A6-A9 fused gather/tcgen05/gate/scatter kernels, A12 completion signal, A13 poll/retire),
+by the C-ABI engine's own event loop (bm_run). lambda* = the highest rate of a load sweep
+(run first, untimed) whose p90 latency stays within the bound (--p90-ms, default 12 ms: the
+paper's flat-region LSTM p90, L489).
+
+value    = requests completed by all ranks / max over ranks of the device time of the K steps
+e2e      = same, through the public API with host buffers: per step the bm_request arrays are
+           submitted from host memory, row descriptors (tokens inside) go host->device from
+           pinned memory on every Schedule call, and all final h rows come back device->host
+roofline = the LSTM cell-step kernel: algorithmic bytes / CUDA-event time of every launch in
+           the timed region, against MEASURED_PEAKS.json
+Multi-GPU (torchrun): one engine per GPU, requests sharded by rank (weak scaling: each rank
+runs its own lambda* Poisson stream), weights broadcast once from rank 0 with NCCL; no
+collective on the per-step path.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from workloads import gen  # noqa: E402
+
+METRIC = "requests/sec at p90-latency bound"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--workload", default="lstm", choices=["lstm", "seq2seq", "tree"])
+    p.add_argument("--reqs", type=int, default=0, help="requests per step (0 = per-workload default)")
+    p.add_argument("--p90-ms", type=float, default=12.0)
+    p.add_argument("--rate", type=float, default=0.0, help="skip the sweep, use this offered rate")
+    p.add_argument("--lookahead", type=int, default=2,
+                   help="schedule when <= k tasks are outstanding (0 = the paper's idle-only)")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=15.0)
+    p.add_argument("--out", default="")
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------------------ workloads
+WL = {
+    "lstm": dict(config="BASELINE configs[1]: 1-layer LSTM h=1024, WMT-like lengths, Poisson arrivals, "
+                        "bmax 512, 1 B200", hidden=1024, layers=1, vocab=32768, reqs=20000),
+    "seq2seq": dict(config="BASELINE configs[2]: Seq2Seq 4+4 layer LSTM h=1024, vocab 32768, greedy "
+                           "decode, encoder/decoder bmax 512/256", hidden=1024, layers=4, vocab=32768,
+                    reqs=4000),
+    "tree": dict(config="BASELINE configs[3]: TreeLSTM h=1024, TreeBank-shaped binary trees, leaf/internal "
+                        "cells batched separately, bmax 64", hidden=1024, layers=1, vocab=32768, reqs=6000),
+}
+
+
+def make_trace(wl, n, rate, seed):
+    if wl == "lstm":
+        return gen.chain_trace(n, WL[wl]["vocab"], seed, rate=rate)
+    if wl == "seq2seq":
+        return gen.seq2seq_trace(n, WL[wl]["vocab"], seed, rate=rate)
+    return gen.tree_trace(n, WL[wl]["vocab"], seed, rate=rate)
+
+
+def make_weights(wl):
+    h, L, V = WL[wl]["hidden"], WL[wl]["layers"], WL[wl]["vocab"]
+    if wl == "lstm":
+        return {"cell": gen.lstm_stack_weights(h, L, V, seed=0)}
+    if wl == "seq2seq":
+        return {"enc": gen.lstm_stack_weights(h, L, V, seed=0),
+                "dec": gen.lstm_stack_weights(h, L, V, seed=1, projection=True)}
+    return {"tree": gen.tree_weights(h, V, seed=0)}
+
+
+def weight_arrays(w):
+    """Flat list of (name, ndarray) views of every weight array (for the NCCL broadcast)."""
+    out = []
+    for k, v in sorted(w.items()):
+        for f in ("W", "b"):
+            if hasattr(v, f):
+                for i, a in enumerate(getattr(v, f)):
+                    out.append((f"{k}.{f}{i}", a))
+        for f in ("E", "W_out", "b_out", "W_leaf", "b_leaf", "U", "b_int"):
+            a = getattr(v, f, None)
+            if a is not None:
+                out.append((f"{k}.{f}", a))
+    return out
+
+
+# ------------------------------------------------------------------------------ engine
+def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, keep=0):
+    h, L, V = WL[wl]["hidden"], WL[wl]["layers"], WL[wl]["vocab"]
+    e = bm.Engine(device=device, hidden=h, pool_layers=L, max_slots=1 << 16, max_requests=max_requests,
+                  schedule_when_outstanding_leq=lookahead, time_kernels=time_kernels, keep_results=keep,
+                  max_decode_len=340)
+    if wl == "lstm":
+        c = w["cell"]
+        cid = e.load_cell(bm.CELL_LSTM, L, V, 512, 0, c.W, c.b, c.E)
+        cells = {gen.CHAIN: (cid, 0)}
+    elif wl == "seq2seq":
+        enc, dec = w["enc"], w["dec"]
+        ce = e.load_cell(bm.CELL_LSTM, L, V, 512, 0, enc.W, enc.b, enc.E)
+        cd = e.load_cell(bm.CELL_LSTM_PROJ, L, V, 256, 1, dec.W, dec.b, dec.E, dec.W_out, dec.b_out)
+        cells = {gen.SEQ2SEQ: (ce, cd)}
+    else:
+        t = w["tree"]
+        lf = e.load_cell(bm.CELL_TREE_LEAF, 1, V, 64, 0, [t.W_leaf], [t.b_leaf], t.E)
+        it = e.load_cell(bm.CELL_TREE_INTERNAL, 1, V, 64, 1, [t.U], [t.b_int])
+        cells = {gen.TREE: (lf, it)}
+    return e, cells
+
+
+def run_trace(e, prepared, n):
+    """Submit a prepared trace and drive it to completion; returns (wall s, latencies s)."""
+    e.submit_many(prepared)
+    t0 = time.perf_counter()
+    done = e.run()
+    t1 = time.perf_counter()
+    comp = e.poll(n + 16)
+    assert done == n and len(comp) == n, (done, len(comp), n)
+    lat = np.array([c.t_done - c.t_arrival for c in comp])
+    return t1 - t0, lat
+
+
+def pct(a, q):
+    return float(np.percentile(a, q)) if len(a) else float("nan")
+
+
+# ------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled DURING the timed region."""
+
+    def __init__(self, device):
+        self.device = device
+        self.samples = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm = [float(s[0]) for s in self.samples if len(s) >= 8 and s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if len(s) >= 8 and s[1].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for s in self.samples:
+            if len(s) >= 8:
+                for i, n in enumerate(names):
+                    if s[4 + i].lower() == "active":
+                        reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------ CPU oracle
+def _oracle_worker(args):
+    os.environ["OMP_NUM_THREADS"] = "1"
+    wl, idx, seed, n = args
+    from oracle import cells
+    w = make_weights(wl)
+    trace = make_trace(wl, n, None, seed)
+    t0 = time.perf_counter()
+    for i in idx:
+        q = trace[i]
+        if wl == "lstm":
+            cells.chain_lstm(w["cell"], q.tokens)
+        elif wl == "seq2seq":
+            cells.seq2seq(w["enc"], w["dec"], q.tokens, q.decode_len)
+        else:
+            cells.tree_lstm(w["tree"], q.tokens, q.left, q.right)
+    return len(idx), time.perf_counter() - t0
+
+
+def cpu_oracle(wl, seconds, seed=1000):
+    """The fp64 oracle (unbatched, step by step) on the host cores over a bounded sample of the
+    same generated requests: one process per core, BLAS pinned to one thread."""
+    import multiprocessing as mp
+    cores = os.cpu_count() or 1
+    # calibrate: one request alone
+    n_est, dt = _oracle_worker((wl, [0, 1], seed, 64))
+    per_req = dt / n_est
+    per_core = max(1, int(seconds / per_req))
+    n = per_core * cores
+    ctx = mp.get_context("fork")
+    t0 = time.perf_counter()
+    with ctx.Pool(cores, initializer=os.environ.__setitem__, initargs=("OMP_NUM_THREADS", "1")) as pool:
+        res = pool.map(_oracle_worker, [(wl, list(range(c * per_core, (c + 1) * per_core)), seed, n)
+                                        for c in range(cores)])
+    wall = time.perf_counter() - t0
+    done = sum(r[0] for r in res)
+    return {"value": done / wall, "unit": "requests/sec", "cores": cores, "kind": "oracle",
+            "sample": f"{done} requests of the same {wl} trace generator (seed {seed}), fp64 numpy, "
+                      f"closed loop, {cores} processes x 1 BLAS thread, {wall:.1f} s wall"}
+
+
+# ------------------------------------------------------------------------------ reference arm
+def reference_arm(a):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    wl = a.workload
+    res = []
+    for s in range(a.warmup + a.steps):
+        r = cpu_oracle(wl, max(2.0, min(a.cpu_seconds, 10.0)), seed=1000 + s)
+        if s >= a.warmup:
+            res.append(r)
+    v = float(np.mean([r["value"] for r in res]))
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "requests/sec", "n_gpus": a.gpus,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": None, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": WL[wl]["config"]},
+            "cpu_baseline": {"value": v, "unit": "requests/sec", "cores": res[0]["cores"], "kind": "oracle",
+                             "sample": res[0]["sample"]},
+            "e2e": {"value": v, "unit": "requests/sec", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------ main arm
+def main():
+    a = parse()
+    if a.impl == "reference":
+        return reference_arm(a)
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    from paper_conf_eurosys_gaoywl18_b200 import bm
+
+    wl = a.workload
+    n_req = a.reqs or WL[wl]["reqs"]
+    # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink), never again
+    w = make_weights(wl)
+    if dist is not None:
+        for name, arr in weight_arrays(w):
+            t = torch.from_numpy(arr).cuda() if rank == 0 else torch.empty(arr.shape, dtype=torch.float32,
+                                                                            device="cuda")
+            dist.broadcast(t, src=0)
+            arr[...] = t.cpu().numpy()
+    e, cells = build_engine(bm, wl, w, local, max_requests=max(n_req, 1 << 15) + 64, lookahead=a.lookahead)
+    stream = torch.cuda.ExternalStream(e.stream(), device=torch.device("cuda", local))
+
+    def barrier():
+        torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+
+    def allmax(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---- calibrate saturation: every request of a trace arrives at t = 0
+    burst = make_trace(wl, n_req, None, seed=7 + rank)
+    pb = e.prepare_requests(burst, cells)
+    run_trace(e, pb, n_req)                      # warm (also JIT of nothing: all AOT)
+    dt, _ = run_trace(e, pb, n_req)
+    mu = n_req / dt
+    # ---- load sweep (open loop), untimed: highest rate whose p90 <= bound
+    curve = []
+    if a.rate > 0:
+        lam_star = a.rate
+    else:
+        lam_star = None
+        for frac in (0.05, 0.1, 0.2, 0.35, 0.5, 0.65, 0.8, 0.9, 1.0, 1.1):
+            lam = frac * mu
+            n_pt = int(max(2000, min(n_req, lam * 0.25)))
+            tr = make_trace(wl, n_pt, lam, seed=100 + rank)
+            p = e.prepare_requests(tr, cells)
+            wall, lat = run_trace(e, p, n_pt)
+            p50, p90, p99 = (allmax(pct(lat, q)) for q in (50, 90, 99))
+            thr = allmax(n_pt / wall)
+            curve.append({"offered": lam, "achieved": n_pt / wall, "p50_ms": p50 * 1e3, "p90_ms": p90 * 1e3,
+                          "p99_ms": p99 * 1e3})
+            if p90 * 1e3 <= a.p90_ms:
+                lam_star = lam
+            elif lam_star is not None:
+                break
+        if lam_star is None:
+            lam_star = 0.05 * mu
+    # ---- timed steps at lambda*
+    trace = make_trace(wl, n_req, lam_star, seed=1000 + rank)
+    prep = e.prepare_requests(trace, cells)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
+    for _ in range(a.warmup):
+        run_trace(e, prep, n_req)
+    e.reset_stats()
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    dev_ms = 0.0
+    lats = []
+    with ClockSampler(local) as clk:
+        for _ in range(a.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            e.submit_many(prep)
+            ev0.record(stream)
+            done = e.run()
+            ev1.record(stream)
+            ev1.synchronize()
+            assert done == n_req
+            dev_ms += ev0.elapsed_time(ev1)
+            comp = e.poll(n_req + 16)
+            lats.append(np.array([c.t_done - c.t_arrival for c in comp]))
+    barrier()
+    st = e.stats()
+    lat = np.concatenate(lats)
+    t_max = allmax(dev_ms / 1e3)
+    total = n_req * a.steps * world
+    value = total / t_max
+    p50, p90, p99 = (allmax(pct(lat, q)) for q in (50, 90, 99))
+    # ---- e2e: public API with host buffers (submit from host, descriptors H2D every Schedule
+    #      call inside bm_run, final h rows D2H), timed on the host clock around the whole thing
+    e2, cells2 = build_engine(bm, wl, w, local, max_requests=n_req + 64, lookahead=a.lookahead,
+                              time_kernels=0, keep=1)
+    L, H = WL[wl]["layers"], WL[wl]["hidden"]
+    hbuf = torch.empty((n_req, L, H), dtype=torch.float32).pin_memory().numpy()
+    prep2 = e2.prepare_requests(trace, cells2)
+    for _ in range(max(1, a.warmup)):
+        fid = e2.submit_many(prep2)
+        e2.run()
+        e2.poll(n_req + 16)
+        e2.read_results_many(fid, n_req, h=hbuf, release=True)
+    barrier()
+    t0 = time.perf_counter()
+    rows0 = e2.stats()["rows"]
+    for _ in range(a.steps):
+        fid = e2.submit_many(prep2)
+        e2.run()
+        e2.poll(n_req + 16)
+        e2.read_results_many(fid, n_req, h=hbuf, release=True)
+    e2e_s = allmax(time.perf_counter() - t0)
+    rows_e2e = (e2.stats()["rows"] - rows0) / a.steps
+    e2e = {"value": total / e2e_s, "unit": "requests/sec",
+           "h2d_bytes_per_step": int(rows_e2e * 16),
+           "d2h_bytes_per_step": int(n_req * L * H * 4)}
+    # ---- roofline of the dominant kernel (the LSTM / tree cell step), live CUDA events
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    achieved = st["timed_bytes"] / (st["timed_ms"] / 1e3) / 1e9 if st["timed_ms"] > 0 else 0.0
+    tflops = st["timed_flops"] / (st["timed_ms"] / 1e3) / 1e12 if st["timed_ms"] > 0 else 0.0
+    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
+            "traffic": None, "kernel": "cell_step_sm100_kernel", "launches": st["timed_launches"],
+            "avg_launch_us": st["timed_ms"] * 1e3 / max(1, st["timed_launches"]),
+            "avg_rows_per_task": st["rows"] / max(1, st["tasks"]), "tensor_tflops": tflops,
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)" if peaks else "fallback 6.65 TB/s"}
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        cpu = cpu_oracle(wl, a.cpu_seconds)
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "requests/sec", "n_gpus": world, "steps": a.steps,
+                "warmup": a.warmup, "ms_per_step": t_max * 1e3 / a.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+                "config": {"workload": WL[wl]["config"], "requests_per_step": n_req,
+                           "offered_rate_per_gpu": lam_star, "p90_bound_ms": a.p90_ms,
+                           "saturation_burst_rate_per_gpu": mu, "lookahead_k": a.lookahead,
+                           "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
+                                 "step (serving)", "parallelism": f"request-sharded x{world}"},
+                "latency_ms": {"p50": p50 * 1e3, "p90": p90 * 1e3, "p99": p99 * 1e3},
+                "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu,
+                "clocks": clk.summary(), "gpu_launches": int(st["kernel_launches"]),
+                "sched_ns_per_task": st["sched_ns"] / max(1, st["tasks"])}
+        s = json.dumps(line)
+        print(s, flush=True)
+        if a.out:
+            with open(a.out, "w") as f:
+                f.write(s + "\n")
+    e.close()
+    e2.close()
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

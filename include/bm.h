@@ -143,6 +143,11 @@ typedef struct {
  * BM_E_FULL (request table full; retry after retiring), BM_E_STATE. */
 bm_status bm_submit(bm_engine* e, const bm_request* r, uint64_t* req_id);
 
+/* Admit n requests in one call (same semantics as n bm_submit calls, stops at the first
+ * failure). *first_id = id of reqs[0]; ids are consecutive. *n_done = requests accepted. */
+bm_status bm_submit_many(bm_engine* e, const bm_request* reqs, int n, uint64_t* first_id,
+                         int* n_done);
+
 /* One scheduler round at the current clock: retire what the device finished, admit due
  * arrivals, and if the worker is idle (<= k outstanding tasks) run Schedule(worker)
  * (Algorithm 1), launching every formed task. *n_tasks = tasks launched (may be 0).
@@ -178,6 +183,12 @@ typedef struct {
  * Errors: BM_E_INVAL (unknown id), BM_E_STATE (not completed / already released). */
 bm_status bm_read_result(bm_engine* e, uint64_t req_id, bm_result* dst);
 bm_status bm_release(bm_engine* e, uint64_t req_id);
+
+/* Bulk result read for the consecutive ids [first_id, first_id + n), all completed and kept:
+ * one device->host copy per contiguous table range. h: [n][pool_layers][hidden] fp32 or
+ * NULL; tokens: [n][max_decode_len] or NULL. Then releases them if release != 0. */
+bm_status bm_read_results_many(bm_engine* e, uint64_t first_id, int n, float* h, int32_t* tokens,
+                               int release);
 
 /* Task log (replay parity, P9): one record per launched task, rows flattened. */
 typedef struct {
@@ -226,7 +237,6 @@ bm_status bm_pool_read(bm_engine* e, int layer, int parity, const int32_t* slots
 bm_status bm_result_rows(bm_engine* e, const int32_t* res_idx, int n, float* h, float* c);
 /* Device feed tokens tok[slot] (decoder) in/out. */
 bm_status bm_tokens(bm_engine* e, const int32_t* slots, int n, int32_t* inout, int write);
-/* Logits of a BM_CELL_LSTM_PROJ step (requires record_logits) for rows' results. */
 
 /* ---------------------------------------------------------------- measurement */
 typedef struct {

@@ -94,11 +94,15 @@ _SIGS = {
     "bm_abi_version": (C.c_int, []),
     "bm_load_cell": (C.c_int, [_P, C.POINTER(CellDesc), C.POINTER(Weights), C.POINTER(C.c_int)]),
     "bm_submit": (C.c_int, [_P, C.POINTER(Request), C.POINTER(C.c_uint64)]),
+    "bm_submit_many": (C.c_int, [_P, C.POINTER(Request), C.c_int, C.POINTER(C.c_uint64),
+                                 C.POINTER(C.c_int)]),
     "bm_schedule_step": (C.c_int, [_P, C.POINTER(C.c_int)]),
     "bm_poll": (C.c_int, [_P, C.POINTER(Completion), C.c_int, C.POINTER(C.c_int)]),
     "bm_run": (C.c_int, [_P, C.POINTER(C.c_int)]),
     "bm_read_result": (C.c_int, [_P, C.c_uint64, C.POINTER(Result)]),
     "bm_release": (C.c_int, [_P, C.c_uint64]),
+    "bm_read_results_many": (C.c_int, [_P, C.c_uint64, C.c_int, C.POINTER(C.c_float),
+                                       C.POINTER(C.c_int32), C.c_int]),
     "bm_read_log": (C.c_int, [_P, C.POINTER(TaskRecord), C.c_int, C.POINTER(C.c_int)]),
     "bm_read_log_rows": (C.c_int, [_P, C.POINTER(RowRecord), C.c_int, C.POINTER(C.c_int)]),
     "bm_cell_step": (C.c_int, [_P, C.c_int, C.POINTER(StepRow), C.c_int, C.c_int]),
@@ -117,6 +121,11 @@ for _name, (_res, _args) in _SIGS.items():
     _f = getattr(lib, _name)
     _f.restype = _res
     _f.argtypes = _args
+
+
+class _Prepared:
+    def __init__(self, arr, toks, lr):
+        self.arr, self.toks, self.lr = arr, toks, lr
 
 
 class BMError(RuntimeError):
@@ -210,6 +219,46 @@ class Engine:
         rid = C.c_uint64()
         _ck(lib.bm_submit(self.h, C.byref(q), C.byref(rid)), "bm_submit")
         return rid.value
+
+    def prepare_requests(self, reqs, cells_for_kind, time_scale: float = 1.0):
+        """Marshal a list of workloads.gen.Request into a bm_request array (kept alive on the
+        returned object) for submit_many. cells_for_kind: {kind: (cell0, cell1)}."""
+        toks = np.ascontiguousarray(np.concatenate([q.tokens for q in reqs]).astype(np.int32))
+        trees = [q for q in reqs if q.left is not None]
+        lr = np.ascontiguousarray(np.concatenate([np.concatenate([q.left, q.right]) for q in trees])
+                                  .astype(np.int32)) if trees else np.zeros(1, np.int32)
+        arr = (Request * len(reqs))()
+        base = toks.ctypes.data
+        lbase = lr.ctypes.data
+        off = loff = 0
+        ip = C.POINTER(C.c_int32)
+        for i, q in enumerate(reqs):
+            c0, c1 = cells_for_kind[q.kind]
+            n = len(q.tokens)
+            a = arr[i]
+            a.kind, a.cell0, a.cell1, a.n = q.kind, c0, c1, n
+            a.tokens = C.cast(base + 4 * off, ip)
+            a.decode_len = q.decode_len
+            if q.left is not None:
+                a.left = C.cast(lbase + 4 * loff, ip)
+                a.right = C.cast(lbase + 4 * (loff + n), ip)
+                loff += 2 * n
+            a.arrival = q.arrival * time_scale
+            a.user_tag = i
+            off += n
+        return _Prepared(arr, toks, lr)
+
+    def submit_many(self, prepared) -> int:
+        first = C.c_uint64()
+        n = C.c_int()
+        _ck(lib.bm_submit_many(self.h, prepared.arr, len(prepared.arr), C.byref(first), C.byref(n)),
+            "bm_submit_many")
+        return first.value
+
+    def read_results_many(self, first_id: int, n: int, h: Optional[np.ndarray] = None,
+                          tokens: Optional[np.ndarray] = None, release: bool = True):
+        _ck(lib.bm_read_results_many(self.h, first_id, n, _fp(h), _ip(tokens), 1 if release else 0),
+            "bm_read_results_many")
 
     def schedule_step(self) -> int:
         n = C.c_int()

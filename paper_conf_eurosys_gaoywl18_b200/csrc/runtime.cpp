@@ -654,6 +654,20 @@ bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
   return BM_OK;
 }
 
+bm_status bm_submit_many(bm_engine* h, const bm_request* reqs, int n, uint64_t* first_id, int* n_done) {
+  if (h == nullptr || reqs == nullptr || n < 0) return BM_E_INVAL;
+  int k = 0;
+  bm_status s = BM_OK;
+  for (; k < n; ++k) {
+    uint64_t id;
+    s = bm_submit(h, reqs + k, &id);
+    if (s != BM_OK) break;
+    if (k == 0 && first_id) *first_id = id;
+  }
+  if (n_done) *n_done = k;
+  return s;
+}
+
 bm_status bm_schedule_step(bm_engine* h, int* n_tasks) {
   if (h == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
@@ -730,17 +744,18 @@ bm_status bm_read_result(bm_engine* h, uint64_t req_id, bm_result* dst) {
   const int ri = static_cast<int>(req_id % e.cfg.max_requests);
   const size_t H = e.H(), L = e.cfg.pool_layers;
   CK(cudaStreamSynchronize(e.stream));
-  if (dst->h) CK(cudaMemcpy(dst->h, e.res_h + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost));
-  if (dst->c) CK(cudaMemcpy(dst->c, e.res_c + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost));
+  if (dst->h) CK(cudaMemcpyAsync(dst->h, e.res_h + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost, e.stream));
+  if (dst->c) CK(cudaMemcpyAsync(dst->c, e.res_c + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost, e.stream));
   if (r.kind == BM_REQ_SEQ2SEQ) {
     const int T = r.n_nodes - r.enc_len;
     if (dst->tokens)
-      CK(cudaMemcpy(dst->tokens, e.res_tok + static_cast<size_t>(ri) * e.cfg.max_decode_len, T * 4,
-                    cudaMemcpyDeviceToHost));
+      CK(cudaMemcpyAsync(dst->tokens, e.res_tok + static_cast<size_t>(ri) * e.cfg.max_decode_len, T * 4,
+                         cudaMemcpyDeviceToHost, e.stream));
     if (dst->logits && e.logits)
-      CK(cudaMemcpy(dst->logits, e.logits + static_cast<size_t>(ri) * e.cfg.max_decode_len * e.logits_vocab,
-                    static_cast<size_t>(T) * e.logits_vocab * 4, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpyAsync(dst->logits, e.logits + static_cast<size_t>(ri) * e.cfg.max_decode_len * e.logits_vocab,
+                         static_cast<size_t>(T) * e.logits_vocab * 4, cudaMemcpyDeviceToHost, e.stream));
   }
+  CK(cudaStreamSynchronize(e.stream));
   return BM_OK;
 }
 
@@ -752,6 +767,40 @@ bm_status bm_release(bm_engine* h, uint64_t req_id) {
   if (!r.done) return BM_E_STATE;
   r.used = false;
   e.n_live_reqs -= 1;
+  return BM_OK;
+}
+
+bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh, int32_t* toks,
+                               int release) {
+  if (h == nullptr || n < 1) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  if (e.sticky_cuda) return BM_E_CUDA;
+  if (!e.device()) return BM_E_STATE;
+  const uint64_t R = e.cfg.max_requests;
+  if (static_cast<uint64_t>(n) > R) return BM_E_INVAL;
+  for (int i = 0; i < n; ++i) {
+    const Request& r = e.reqs[(first_id + i) % R];
+    if (!r.used || r.id != first_id + i) return BM_E_INVAL;
+    if (!r.done) return BM_E_STATE;
+  }
+  const size_t LH = e.H() * e.cfg.pool_layers;
+  const size_t D = e.cfg.max_decode_len;
+  int done = 0;
+  while (done < n) {  // contiguous table ranges (the table is a ring)
+    const size_t ri = (first_id + done) % R;
+    const int len = static_cast<int>(std::min<uint64_t>(n - done, R - ri));
+    if (hh) CK(cudaMemcpyAsync(hh + done * LH, e.res_h + ri * LH, len * LH * 4, cudaMemcpyDeviceToHost, e.stream));
+    if (toks) CK(cudaMemcpyAsync(toks + done * D, e.res_tok + ri * D, len * D * 4, cudaMemcpyDeviceToHost, e.stream));
+    done += len;
+  }
+  CK(cudaStreamSynchronize(e.stream));
+  if (release) {
+    for (int i = 0; i < n; ++i) {
+      Request& r = e.reqs[(first_id + i) % R];
+      r.used = false;
+      e.n_live_reqs -= 1;
+    }
+  }
   return BM_OK;
 }
 
@@ -805,18 +854,21 @@ static bm_status pool_io(Engine& e, int layer, int parity, const int32_t* slots,
   CK(cudaMalloc(&ds, n * 4));
   CK(cudaMalloc(&dh, n * H * 4));
   CK(cudaMalloc(&dc, n * H * 4));
-  CK(cudaMemcpy(ds, slots, n * 4, cudaMemcpyHostToDevice));
+  // every copy is ordered on the engine stream (a pageable cudaMemcpy on the legacy stream
+  // may still be in flight when a kernel on the non-blocking engine stream starts)
+  CK(cudaMemcpyAsync(ds, slots, n * 4, cudaMemcpyHostToDevice, e.stream));
   if (write) {
-    if (h) CK(cudaMemcpy(dh, h, n * H * 4, cudaMemcpyHostToDevice));
-    if (c) CK(cudaMemcpy(dc, c, n * H * 4, cudaMemcpyHostToDevice));
+    if (h) CK(cudaMemcpyAsync(dh, h, n * H * 4, cudaMemcpyHostToDevice, e.stream));
+    if (c) CK(cudaMemcpyAsync(dc, c, n * H * 4, cudaMemcpyHostToDevice, e.stream));
   }
   void* hp = static_cast<char*>(e.h_layer(layer)) + static_cast<size_t>(parity) * e.cfg.max_slots * H * e.elem();
   CK(launch_pool_io(hp, e.c_layer(layer), ds, n, static_cast<int>(H), h ? dh : nullptr,
                     c ? dc : nullptr, write, e.cfg.precision == BM_PREC_BF16, e.stream));
   CK(cudaStreamSynchronize(e.stream));
   if (!write) {
-    if (h) CK(cudaMemcpy(h, dh, n * H * 4, cudaMemcpyDeviceToHost));
-    if (c) CK(cudaMemcpy(c, dc, n * H * 4, cudaMemcpyDeviceToHost));
+    if (h) CK(cudaMemcpyAsync(h, dh, n * H * 4, cudaMemcpyDeviceToHost, e.stream));
+    if (c) CK(cudaMemcpyAsync(c, dc, n * H * 4, cudaMemcpyDeviceToHost, e.stream));
+    CK(cudaStreamSynchronize(e.stream));
   }
   cudaFree(ds);
   cudaFree(dh);
@@ -845,9 +897,10 @@ bm_status bm_result_rows(bm_engine* h, const int32_t* res_idx, int n, float* hh,
   CK(cudaStreamSynchronize(e.stream));
   for (int i = 0; i < n; ++i) {
     if (res_idx[i] < 0 || res_idx[i] >= e.cfg.max_requests) return BM_E_INVAL;
-    if (hh) CK(cudaMemcpy(hh + i * LH, e.res_h + res_idx[i] * LH, LH * 4, cudaMemcpyDeviceToHost));
-    if (cc) CK(cudaMemcpy(cc + i * LH, e.res_c + res_idx[i] * LH, LH * 4, cudaMemcpyDeviceToHost));
+    if (hh) CK(cudaMemcpyAsync(hh + i * LH, e.res_h + res_idx[i] * LH, LH * 4, cudaMemcpyDeviceToHost, e.stream));
+    if (cc) CK(cudaMemcpyAsync(cc + i * LH, e.res_c + res_idx[i] * LH, LH * 4, cudaMemcpyDeviceToHost, e.stream));
   }
+  CK(cudaStreamSynchronize(e.stream));
   return BM_OK;
 }
 
@@ -858,9 +911,10 @@ bm_status bm_tokens(bm_engine* h, const int32_t* slots, int n, int32_t* inout, i
   CK(cudaStreamSynchronize(e.stream));
   for (int i = 0; i < n; ++i) {
     if (slots[i] < 0 || slots[i] >= e.cfg.max_slots) return BM_E_INVAL;
-    if (write) CK(cudaMemcpy(e.tok + slots[i], inout + i, 4, cudaMemcpyHostToDevice));
-    else CK(cudaMemcpy(inout + i, e.tok + slots[i], 4, cudaMemcpyDeviceToHost));
+    if (write) CK(cudaMemcpyAsync(e.tok + slots[i], inout + i, 4, cudaMemcpyHostToDevice, e.stream));
+    else CK(cudaMemcpyAsync(inout + i, e.tok + slots[i], 4, cudaMemcpyDeviceToHost, e.stream));
   }
+  CK(cudaStreamSynchronize(e.stream));
   return BM_OK;
 }
 
