@@ -214,26 +214,40 @@ def _oracle_worker(args):
     return len(idx), time.perf_counter() - t0
 
 
+def _cost(q):
+    """Cell steps of one request (the oracle's work unit)."""
+    return len(q.tokens) + q.decode_len if q.left is None else len(q.left)
+
+
 def cpu_oracle(wl, seconds, seed=1000):
     """The fp64 oracle (unbatched, step by step) on the host cores over a bounded sample of the
-    same generated requests: one process per core, BLAS pinned to one thread."""
+    same generated requests: one process per core, BLAS pinned to one thread. The sample is the
+    first requests of the trace whose total cell steps fit ~`seconds` of work per core."""
     import multiprocessing as mp
     cores = os.cpu_count() or 1
-    # calibrate: one request alone
-    n_est, dt = _oracle_worker((wl, [0, 1], seed, 64))
-    per_req = dt / n_est
-    per_core = max(1, int(seconds / per_req))
-    n = per_core * cores
+    trace = make_trace(wl, 20000, None, seed)
+    # calibrate the cost of one cell step on this host
+    probe = [i for i in range(len(trace)) if _cost(trace[i]) >= 8][:1]
+    n_est, dt = _oracle_worker((wl, probe, seed, 20000))
+    per_step = dt / _cost(trace[probe[0]])
+    budget = seconds * cores / per_step
+    idx, tot = [], 0
+    for i, q in enumerate(trace):
+        if tot + _cost(q) > budget and idx:
+            break
+        idx.append(i)
+        tot += _cost(q)
+    chunks = [idx[c::cores] for c in range(cores)]
     ctx = mp.get_context("fork")
     t0 = time.perf_counter()
-    with ctx.Pool(cores, initializer=os.environ.__setitem__, initargs=("OMP_NUM_THREADS", "1")) as pool:
-        res = pool.map(_oracle_worker, [(wl, list(range(c * per_core, (c + 1) * per_core)), seed, n)
-                                        for c in range(cores)])
+    with ctx.Pool(cores) as pool:
+        res = pool.map(_oracle_worker, [(wl, ch, seed, 20000) for ch in chunks if ch])
     wall = time.perf_counter() - t0
     done = sum(r[0] for r in res)
     return {"value": done / wall, "unit": "requests/sec", "cores": cores, "kind": "oracle",
-            "sample": f"{done} requests of the same {wl} trace generator (seed {seed}), fp64 numpy, "
-                      f"closed loop, {cores} processes x 1 BLAS thread, {wall:.1f} s wall"}
+            "sample": f"first {done} requests ({tot} cell steps) of the {wl} trace generator "
+                      f"(seed {seed}), fp64 numpy, closed loop, {cores} processes x 1 BLAS thread, "
+                      f"{wall:.1f} s wall"}
 
 
 # ------------------------------------------------------------------------------ reference arm

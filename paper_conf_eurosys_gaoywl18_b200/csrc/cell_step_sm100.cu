@@ -174,6 +174,16 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
 
+// Diagnostics (BM_PHASE_DUMP): %globaltimer of one thread at phase boundaries of each CTA.
+__device__ __forceinline__ void phase_mark(const StepArgs& p, int i) {
+  if (p.phase != nullptr) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+    p.phase[cta * 8 + i] = t;
+  }
+}
+
 // ------------------------------------------------------------------ row sources (A6)
 // Pointer to the first element of a row's operand segment `seg`, or nullptr for a zero row.
 template <int EPI>
@@ -237,6 +247,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
 
   // ---- setup
+  if (tid == 0) phase_mark(p, 0);
   if (tid == 0) {
     for (int s = 0; s < kStages; ++s) {
       mbar_init(full0 + 8 * s, kProducerThreads);
@@ -268,6 +279,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  if (tid == 0) phase_mark(p, 1);
 
   if (warp < 8) {
     // ================================================================ producers (A6, A7)
@@ -335,6 +347,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (warp < 8) {
     mbar_wait(done_bar, 0);
     tc_fence_after();
+    if (tid == 0) phase_mark(p, 2);
     const int q = warp & 3;
     const int row = 32 * q + lane;
     for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
@@ -396,6 +409,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else {
     // ============================================================ split-K reduction + gates (A9)
     cluster_sync();
+    if (tid == 0) phase_mark(p, 3);
     const int S = p.S;
     uint32_t peer[8];
     for (int s = 0; s < S; ++s) peer[s] = mapa(smem_u32(P), s);
@@ -456,7 +470,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
+    if (tid == 0) phase_mark(p, 4);
     cluster_sync();  // peers may still read this CTA's partials until here
+    if (tid == 0) phase_mark(p, 5);
   }
 
   if (warp == 8) {

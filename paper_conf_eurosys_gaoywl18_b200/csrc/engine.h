@@ -140,6 +140,7 @@ struct Engine {
   unsigned long long* signal_host = nullptr;   // pinned, mapped
   unsigned long long* signal_dev = nullptr;
   RowDesc* direct_rows = nullptr;  // bm_cell_step rows (device)
+  unsigned long long* phase_dev = nullptr;  // BM_PHASE_DUMP diagnostics
   std::vector<TimedLaunch> ev_pool;
   int ev_head = 0;
 

@@ -56,6 +56,7 @@ struct StepArgs {
   int32_t* res_tok;           // [max_requests][max_decode]
   int max_decode;
   float* logits;              // debug [max_requests][max_decode][V] or null
+  unsigned long long* phase;  // diagnostics: per-CTA %globaltimer at phase boundaries, or null
 };
 
 // bf16 / tcgen05 path (cell_step_sm100.cu). tmW: TMA map of the packed bf16 weights.

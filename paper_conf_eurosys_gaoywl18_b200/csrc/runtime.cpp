@@ -7,6 +7,8 @@
 // (§5 "Asynchronous Completion Notification", L393-L395); bm_poll / the run loop compare the
 // counter against the in-progress FIFO and retire finished tasks in order.
 #include <cuda_bf16.h>
+#include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -129,6 +131,7 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
   a.res_tok = e.res_tok;
   a.max_decode = e.cfg.max_decode_len;
   a.logits = (proj && e.logits != nullptr) ? e.logits : nullptr;
+  a.phase = e.phase_dev;
   TimedLaunch* tl = nullptr;
   if (e.cfg.time_kernels && !e.ev_pool.empty()) {
     const int i = e.ev_head;
@@ -387,6 +390,7 @@ static void free_device(Engine& e) {
   cudaFree(e.done_ctas);
   cudaFree(e.ring_dev);
   cudaFree(e.direct_rows);
+  cudaFree(e.phase_dev);
   if (e.ring_host) cudaFreeHost(e.ring_host);
   if (e.signal_host) cudaFreeHost(e.signal_host);
   for (TimedLaunch& t : e.ev_pool) {
@@ -835,9 +839,28 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
     if ((rows[i].flags >> 8) >= e.cfg.max_requests) return BM_E_INVAL;
   }
   CK(cudaMemcpyAsync(e.direct_rows, rows, sizeof(RowDesc) * b, cudaMemcpyHostToDevice, e.stream));
+  // diagnostics: BM_PHASE_DUMP=<file> records per-CTA phase timestamps of every direct step
+  static const char* dump = getenv("BM_PHASE_DUMP");
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 8 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 8 * 4096, e.stream));
   bm_status s = launch_cell(e, c, e.direct_rows, b, nullptr);
   if (s != BM_OK) return s;
-  if (!async) CK(cudaStreamSynchronize(e.stream));
+  if (!async || e.phase_dev) CK(cudaStreamSynchronize(e.stream));
+  if (e.phase_dev) {
+    std::vector<unsigned long long> h(8 * 4096);
+    CK(cudaMemcpy(h.data(), e.phase_dev, h.size() * 8, cudaMemcpyDeviceToHost));
+    FILE* f = fopen(dump, "a");
+    if (f) {
+      fprintf(f, "step b=%d cell=%d\n", b, cell_id);
+      for (int i = 0; i < 4096; ++i)
+        if (h[i * 8]) {
+          fprintf(f, "%d", i);
+          for (int k = 0; k < 8; ++k) fprintf(f, " %llu", h[i * 8 + k]);
+          fprintf(f, "\n");
+        }
+      fclose(f);
+    }
+  }
   return BM_OK;
 }
 

@@ -89,7 +89,7 @@ def test_lstm_stack_step_parity(prec):
 def test_tree_cells_parity(prec, b):
     rng = np.random.default_rng(b)
     h, V = 1024, 300
-    e, (leaf, intern), w = tree_engine(h, V, prec, bmax=512, max_slots=2048, max_requests=1024)
+    e, (leaf, intern), w = tree_engine(h, V, prec, bmax=512, max_slots=2048, max_requests=2048)
     # leaves -> slots A ; internal nodes combine random pairs of them -> slots B
     A = _slots(rng, 2 * b, 1024)
     toks = rng.integers(3, V, size=2 * b)

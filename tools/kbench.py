@@ -1,0 +1,80 @@
+"""Kernel micro-benchmark: one batched cell step (bm_cell_step, async) at fixed b, timed with
+CUDA events on the engine stream over many back-to-back launches. Reports us/launch,
+algorithmic GB/s and TFLOP/s per b. Used for the roofline sweep and under ncu."""
+import argparse
+import json
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--cell", default="lstm", choices=["lstm", "leaf", "internal", "proj"])
+    ap.add_argument("--b", default="1,16,64,128,256,512")
+    ap.add_argument("--iters", type=int, default=200)
+    ap.add_argument("--fp32", action="store_true")
+    ap.add_argument("--out", default="")
+    a = ap.parse_args()
+    import torch
+    from paper_conf_eurosys_gaoywl18_b200 import bm
+    from workloads import gen
+    H, V = 1024, 32768
+    prec = bm.PREC_FP32 if a.fp32 else bm.PREC_BF16
+    bf = not a.fp32
+    e = bm.Engine(precision=prec, hidden=H, pool_layers=1, max_slots=8192, max_requests=8192,
+                  max_decode_len=4)
+    if a.cell in ("lstm", "proj"):
+        w = gen.lstm_stack_weights(H, 1, V, 0, projection=a.cell == "proj", bf16=bf)
+        kind = bm.CELL_LSTM_PROJ if a.cell == "proj" else bm.CELL_LSTM
+        cid = e.load_cell(kind, 1, V, 512, 0, w.W, w.b, w.E, w.W_out, w.b_out)
+        G, K, rows_w = 4, 2 * H, 4 * H
+    else:
+        t = gen.tree_weights(H, V, 0, bf16=bf)
+        leaf = e.load_cell(bm.CELL_TREE_LEAF, 1, V, 512, 0, [t.W_leaf], [t.b_leaf], t.E)
+        intern = e.load_cell(bm.CELL_TREE_INTERNAL, 1, V, 512, 1, [t.U], [t.b_int])
+        cid = leaf if a.cell == "leaf" else intern
+        G, K = (3, H) if a.cell == "leaf" else (5, 2 * H)
+        rows_w = G * H
+    stream = torch.cuda.ExternalStream(e.stream())
+    rng = np.random.default_rng(0)
+    out = []
+    el = 2 if bf else 4
+    for b in [int(x) for x in a.b.split(",")]:
+        slots = rng.choice(8192, size=b, replace=False).astype(np.int32)
+        if a.cell == "internal":
+            kids = rng.choice(8192, size=2 * b, replace=False).astype(np.int32)
+            rows = np.stack([kids[:b], kids[b:], slots, np.zeros(b)], 1)
+        else:
+            toks = rng.integers(3, V, size=b)
+            rows = np.stack([toks, np.zeros(b), slots, (np.arange(b) % 2) * bm.ROW_PARITY], 1)
+        for _ in range(5):
+            e.cell_step(cid, rows, sync=False)
+        torch.cuda.synchronize()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for _ in range(a.iters):
+            e.cell_step(cid, rows, sync=False)
+        ev1.record(stream)
+        ev1.synchronize()
+        us = ev0.elapsed_time(ev1) * 1e3 / a.iters
+        if a.cell == "proj":
+            # LSTM layer + projection per call; report the sum
+            byts = (rows_w * K * el + b * 14336) + (V * H * el + b * (2 * H + 8))
+            flops = 2 * b * K * rows_w + 2 * b * H * V
+        else:
+            per_row = K * el + H * el + H * 4 + (H * 4 if a.cell == "lstm" else 2 * H * 4 if a.cell == "internal" else 0)
+            byts = rows_w * K * el + rows_w * 4 + b * per_row
+            flops = 2 * b * K * rows_w
+        r = {"cell": a.cell, "b": b, "us": us, "GBps": byts / us / 1e3, "TFLOPs": flops / us / 1e6}
+        print(json.dumps(r), flush=True)
+        out.append(r)
+    if a.out:
+        json.dump(out, open(a.out, "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()

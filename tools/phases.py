@@ -1,0 +1,25 @@
+"""Summarise BM_PHASE_DUMP files: per-phase durations (us) over the CTAs of each step.
+Phases: 0 start, 1 setup done, 2 MMA done (main loop), 3 cluster barrier 1, 4 reduce+epilogue,
+5 final cluster barrier."""
+import sys
+
+import numpy as np
+
+steps = []
+cur = None
+for line in open(sys.argv[1]):
+    if line.startswith("step"):
+        cur = {"hdr": line.strip(), "rows": []}
+        steps.append(cur)
+    else:
+        v = [int(x) for x in line.split()]
+        cur["rows"].append(v[1:7])
+for st in steps[-3:]:
+    a = np.array(st["rows"], dtype=np.float64)
+    t0 = a[:, 0].min()
+    print(st["hdr"], "ctas", len(a), "span_us %.2f" % ((a[:, 5].max() - t0) / 1e3))
+    names = ["start", "setup", "mainloop", "bar1", "reduce", "bar2"]
+    print("  start offsets us: min %.2f med %.2f max %.2f" % tuple((np.percentile(a[:, 0] - t0, q) / 1e3) for q in (0, 50, 100)))
+    for k in range(1, 6):
+        d = (a[:, k] - a[:, k - 1]) / 1e3
+        print("  %-8s us: min %.2f med %.2f max %.2f" % (names[k], d.min(), np.median(d), d.max()))
