@@ -77,10 +77,12 @@ typedef struct {
   int keep_results;          /* 1: results stay readable until bm_release; 0: auto-free  */
   int record_logits;         /* debug: keep every decode step's logits (parity tests)     */
   int time_kernels;          /* 1: CUDA-event time every cell-step launch (bench roofline)*/
+  int record_log;            /* 1: keep the task log for bm_read_log (default 1)          */
 } bm_config;
 
 /* Fill *cfg with defaults: device 0, BF16, WALL, hidden 1024, 1 layer, 65536 slots,
- * 65536 requests, MaxTasksToSubmit 5, Min 1, k 0, max_decode_len 512, keep_results 0. */
+ * 65536 requests, MaxTasksToSubmit 5, Min 1, k 0, max_decode_len 512, keep_results 0,
+ * record_log 1. */
 void bm_config_default(bm_config* cfg);
 
 /* ---------------------------------------------------------------- cells (bm_load_cell) */

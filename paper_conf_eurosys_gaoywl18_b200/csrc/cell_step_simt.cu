@@ -257,6 +257,28 @@ __global__ void pack_rows_kernel(const float* __restrict__ src, void* dst, float
   }
 }
 
+// fp32 paper layout -> bf16 "stage tiles" for the tcgen05 kernel: tile t of tile_rows packed
+// rows (packed row n = u * G + g <-> paper row g * H + u; G = 1: identity, the projection), and
+// 64-column K block kc, stored contiguously (tile_rows x 128 B) in the 128B-swizzled K-major
+// layout the UMMA shared-memory descriptor expects: 16-byte chunk j of row r sits at chunk
+// position j ^ (r % 8). One pipeline stage of the kernel is then ONE contiguous bulk copy.
+__global__ void pack_tiles_kernel(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst,
+                                  int G, int H, int K, int tile_rows, int n_rows) {
+  const size_t n = static_cast<size_t>(n_rows) * K;
+  const int kblocks = K / 64;
+  for (size_t e = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; e < n;
+       e += static_cast<size_t>(gridDim.x) * blockDim.x) {
+    const int row = static_cast<int>(e / K);   // packed row
+    const int k = static_cast<int>(e % K);
+    const int src_row = G == 1 ? row : (row % G) * H + row / G;
+    const int t = row / tile_rows, r = row % tile_rows;
+    const int kc = k / 64, j = (k % 64) / 8, el = k % 8;
+    const size_t off = ((static_cast<size_t>(t) * kblocks + kc) * tile_rows + r) * 64 +
+                       ((j ^ (r & 7)) * 8) + el;
+    dst[off] = __float2bfloat16_rn(src[static_cast<size_t>(src_row) * K + k]);
+  }
+}
+
 __global__ void convert_kernel(const float* __restrict__ src, void* dst, size_t n, int bf16) {
   for (size_t e = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; e < n;
        e += static_cast<size_t>(gridDim.x) * blockDim.x) {
@@ -315,6 +337,12 @@ cudaError_t launch_cell_step_simt(const StepArgs& a, cudaStream_t st) {
 cudaError_t launch_pack_rows(const float* src, void* dst, float* bias_dst, const float* bias_src,
                              int G, int H, int K, int bf16, cudaStream_t st) {
   pack_rows_kernel<<<1184, 256, 0, st>>>(src, dst, bias_dst, bias_src, G, H, K, bf16);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pack_tiles(const float* src, void* dst, int G, int H, int K, int tile_rows,
+                              int n_rows, cudaStream_t st) {
+  pack_tiles_kernel<<<1184, 256, 0, st>>>(src, static_cast<__nv_bfloat16*>(dst), G, H, K, tile_rows, n_rows);
   return cudaGetLastError();
 }
 

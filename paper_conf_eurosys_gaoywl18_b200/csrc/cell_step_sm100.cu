@@ -32,13 +32,16 @@
 namespace bm {
 namespace {
 
-constexpr int kStages = 4;
+constexpr int kMaxStages = 8;           // pipeline depth cap
+constexpr int kTailBytes = 5120;        // row-source table [2][256] + barriers, at smem offset 0
 constexpr int kBK = 64;                 // K elements per stage (128 B of bf16 = one SW128 atom)
-constexpr int kProducerThreads = 256;   // warps 0-7
-constexpr int kThreads = kProducerThreads + 32;
+constexpr int kProducerThreads = 256;   // warps 0-7: activation gather (cp.async)
+constexpr int kMmaWarp = 8;             // warp 8: TMEM alloc + tcgen05.mma issue
+constexpr int kTmaWarp = 9;             // warp 9: weight TMA stream
+constexpr int kThreads = kProducerThreads + 64;
 constexpr int kMaxCols = 256;           // batch columns per CTA (MMA N <= 256)
 constexpr int kWStageBytes = 128 * 128; // 128 weight rows x 128 B
-constexpr int kLag = 2;                 // cp.async groups in flight per producer thread
+constexpr int kMaxS = 4;                // max split-K cluster size (K = 2h = 2048 -> 4 x 512)
 
 // ------------------------------------------------------------------ PTX helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -69,12 +72,11 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   while (!mbar_try_wait(bar, parity)) {
   }
 }
-__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar,
-                                            int c0, int c1) {
+// Contiguous global -> shared bulk copy (TMA engine), completion counted on an mbarrier.
+__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
   asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1)
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+      "l"(src), "r"(bytes), "r"(bar)
       : "memory");
 }
 __device__ __forceinline__ void cp_async_16(uint32_t dst, const void* src, uint32_t src_bytes) {
@@ -86,6 +88,19 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+// wait until at most n of this thread's cp.async groups are pending (n is runtime, <= 7)
+__device__ __forceinline__ void cp_async_wait_dyn(int n) {
+  switch (n) {
+    case 0: cp_async_wait<0>(); break;
+    case 1: cp_async_wait<1>(); break;
+    case 2: cp_async_wait<2>(); break;
+    case 3: cp_async_wait<3>(); break;
+    case 4: cp_async_wait<4>(); break;
+    case 5: cp_async_wait<5>(); break;
+    case 6: cp_async_wait<6>(); break;
+    default: cp_async_wait<7>(); break;
+  }
 }
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -110,17 +125,26 @@ __device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
   return r;
 }
+__device__ __forceinline__ void st_cluster_f32(uint32_t addr, float v) {
+  asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void named_bar(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
 __device__ __forceinline__ float ld_cluster_f32(uint32_t addr) {
   float v;
-  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr));
   return v;
 }
 __device__ __forceinline__ float4 ld_cluster_v4(uint32_t addr) {
   float4 v;
   asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
                : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-               : "r"(addr)
-               : "memory");
+               : "r"(addr));
   return v;
 }
 
@@ -172,6 +196,23 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
+// Shared-memory plan (identical on host and device). Small tasks (npad <= 128) keep the
+// footprint near 100 KB so two CTAs fit per SM (the next launch's CTAs can start under PDL while
+// this one drains); larger tasks take ~200 KB. Stage depth matters little (the per-SM ingest
+// rate, not latency, bounds the stream: tools/ingest_bench.cu), so the budget decides it.
+__host__ __device__ __forceinline__ int stage_bytes(int npad) { return kWStageBytes + npad * 128; }
+__host__ __device__ __forceinline__ int stages_for(int npad) {
+  const int budget = npad <= 128 ? 96 * 1024 : 192 * 1024;
+  const int n = budget / stage_bytes(npad);
+  return n < kMaxStages ? (n < 2 ? 2 : n) : kMaxStages;
+}
+// stage ring, reused after the main loop for the partial / logits tile (<= 129 x npad fp32)
+__host__ __device__ __forceinline__ int region_bytes(int npad) {
+  const int a = stages_for(npad) * stage_bytes(npad);
+  const int b = 129 * npad * 4 + 4 * 128 * 4;
+  return a > b ? a : b;
+}
+
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
 
 // Diagnostics (BM_PHASE_DUMP): %globaltimer of one thread at phase boundaries of each CTA.
@@ -216,9 +257,9 @@ __device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const
 // ------------------------------------------------------------------ the kernel
 template <int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
-    cell_step_sm100_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ StepArgs p) {
+    cell_step_sm100_kernel(const __grid_constant__ StepArgs p) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+  uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
@@ -232,60 +273,65 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int npad = (ncols + 15) & ~15;
   const int nk = p.kslice / kBK;
   const int k_begin = static_cast<int>(rank) * p.kslice;
+  const int kStages = p.max_stages > 0 ? min(p.max_stages, stages_for(npad)) : stages_for(npad);
 
-  // shared memory carve-up
+  // shared memory: [tail: row sources + barriers][stage ring: W tiles | X tiles]
+  const __nv_bfloat16** src_tab = reinterpret_cast<const __nv_bfloat16**>(base);  // [2][256]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(base + 2 * kMaxCols * sizeof(void*));
+  const uint32_t full0 = smem_u32(bars);
+  const uint32_t empty0 = smem_u32(bars + kMaxStages);
+  const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 1);
+  int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
+  uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
   uint8_t* w_st = smem;                                   // kStages x 16 KB
   uint8_t* x_st = smem + kStages * kWStageBytes;          // kStages x npad x 128 B
   const int x_stage_bytes = npad * 128;
-  uint8_t* tail = x_st + kStages * x_stage_bytes;
-  const __nv_bfloat16** src_tab = reinterpret_cast<const __nv_bfloat16**>(tail);  // [2][256]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(tail + 2 * kMaxCols * sizeof(void*));
-  const uint32_t full0 = smem_u32(bars);
-  const uint32_t empty0 = smem_u32(bars + kStages);
-  const uint32_t done_bar = smem_u32(bars + 2 * kStages);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kStages + 1);
-  int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
 
-  // ---- setup
+  // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
   if (tid == 0) {
-    for (int s = 0; s < kStages; ++s) {
-      mbar_init(full0 + 8 * s, kProducerThreads);
+    for (int s = 0; s < kMaxStages; ++s) {
+      mbar_init(full0 + 8 * s, kProducerThreads + 1);  // gather threads + the TMA thread
       mbar_init(empty0 + 8 * s, 1);
     }
     mbar_init(done_bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
   }
-  if (warp == 8) {
+  if (warp == kMmaWarp) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                      smem_u32(tmem_slot)),
                  "r"(256)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
-  for (int c = tid; c < kMaxCols; c += kThreads) {
-    const __nv_bfloat16* s0 = nullptr;
-    const __nv_bfloat16* s1 = nullptr;
-    if (c < ncols) {
-      const RowDesc r = p.rows[col0 + c];
-      s0 = seg_src<EPI>(p, r, 0);
-      if (p.K1 > 0) s1 = seg_src<EPI>(p, r, 1);
-    }
-    src_tab[c] = s0;
-    src_tab[kMaxCols + c] = s1;
-  }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_launch_dependents();  // the next launch may start its own setup + weight stream now
   if (tid == 0) phase_mark(p, 1);
 
   if (warp < 8) {
-    // ================================================================ producers (A6, A7)
+    // ================================================================ activation gather (A6)
+    pdl_wait();  // rows, pool h/c and feed tokens are written by earlier launches / copies
+    for (int c = tid; c < kMaxCols; c += kProducerThreads) {
+      const __nv_bfloat16* s0 = nullptr;
+      const __nv_bfloat16* s1 = nullptr;
+      if (c < ncols) {
+        const RowDesc r = p.rows[col0 + c];
+        s0 = seg_src<EPI>(p, r, 0);
+        if (p.K1 > 0) s1 = seg_src<EPI>(p, r, 1);
+      }
+      src_tab[c] = s0;
+      src_tab[kMaxCols + c] = s1;
+    }
+    named_bar(1, kProducerThreads);
+    // Every stage's cp.async group stays in flight until the ring is full; a stage is handed
+    // to the MMA (full barrier) once its group has landed and been made visible to the
+    // async proxy. lag = stages - 1 keeps the whole ring in flight without deadlock.
     const __nv_bfloat16* dummy = static_cast<const __nv_bfloat16*>(p.E != nullptr ? p.E : p.h_pool);
-    const int wbytes = tile_rows * 128;
-    const int wrow0 = blockIdx.y * tile_rows;
+    const int lag = min(kStages - 1, 7);
     for (int kb = 0; kb < nk; ++kb) {
       const int s = kb % kStages;
       const int round = kb / kStages;
@@ -293,10 +339,6 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int k = k_begin + kb * kBK;
       const int seg = k >= p.K0 ? 1 : 0;
       const int kk = k - seg * p.K0;
-      if (tid == 0) {
-        mbar_expect_tx(full0 + 8 * s, wbytes);
-        tma_load_2d(smem_u32(w_st + s * kWStageBytes), &tmW, full0 + 8 * s, k, wrow0);
-      }
       const uint32_t xs = smem_u32(x_st + s * x_stage_bytes);
       const __nv_bfloat16** tab = src_tab + seg * kMaxCols;
       for (int q = tid; q < npad * 8; q += kProducerThreads) {
@@ -311,15 +353,35 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
       cp_async_commit();
-      if (kb >= kLag) {
-        cp_async_wait<kLag>();
+      if (kb >= lag) {
+        cp_async_wait_dyn(lag);
         fence_proxy_async();
-        mbar_arrive(full0 + 8 * ((kb - kLag) % kStages));
+        mbar_arrive(full0 + 8 * ((kb - lag) % kStages));
       }
     }
     cp_async_wait<0>();
     fence_proxy_async();
-    for (int kb = max(0, nk - kLag); kb < nk; ++kb) mbar_arrive(full0 + 8 * (kb % kStages));
+    for (int kb = max(0, nk - lag); kb < nk; ++kb) mbar_arrive(full0 + 8 * (kb % kStages));
+  } else if (warp == kTmaWarp) {
+    // ================================================================ weight stream (A7)
+    // Weights are read-only: streaming starts before griddepcontrol.wait (PDL overlap).
+    if (lane == 0) {
+      const int wbytes = tile_rows * 128;
+      const int kblocks = (p.K0 + p.K1) / kBK;
+      const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
+                            (static_cast<size_t>(blockIdx.y) * kblocks + k_begin / kBK) * wbytes;
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % kStages;
+        const int round = kb / kStages;
+        if (round > 0) mbar_wait(empty0 + 8 * s, (round - 1) & 1);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(full0 + 8 * s),
+                     "r"(wbytes)
+                     : "memory");
+        bulk_load(smem_u32(w_st + s * kWStageBytes), wsrc + static_cast<size_t>(kb) * wbytes, wbytes,
+                  full0 + 8 * s);
+      }
+    }
+    __syncwarp();
   } else {
     // ================================================================ MMA issuer (A8)
     const uint32_t idesc = idesc_bf16(128, npad);
@@ -327,6 +389,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int s = kb % kStages;
       mbar_wait(full0 + 8 * s, (kb / kStages) & 1);
       tc_fence_after();
+      if (lane == 0 && kb == 0) phase_mark(p, 6);
+      if (lane == 0 && kb == nk - 1) phase_mark(p, 7);
       if (lane == 0) {
         const uint64_t a = sdesc_sw128(smem_u32(w_st + s * kWStageBytes));
         const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes));
@@ -340,30 +404,30 @@ __global__ void __launch_bounds__(kThreads, 1)
       __syncwarp();
     }
   }
-
-  // ================================================================ accumulators -> smem
-  float* P = reinterpret_cast<float*>(smem);  // reuses the (drained) stage buffers
-  const int pitch = EPI == EPI_PROJ ? 129 : 128;
   if (warp < 8) {
     mbar_wait(done_bar, 0);
     tc_fence_after();
     if (tid == 0) phase_mark(p, 2);
-    const int q = warp & 3;
-    const int row = 32 * q + lane;
-    for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
-      float v[32];
-      tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
-#pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        if (c0 + i < npad) P[(c0 + i) * pitch + row] = v[i];
-      }
-    }
   }
-  tc_fence_before();
+  const int q = warp & 3;
+  const int trow = 32 * q + lane;  // TMEM lane = tile (weight / vocab) row of this thread
 
   if constexpr (EPI == EPI_PROJ) {
     // ============================================================ projection + argmax (A10)
+    float* P = reinterpret_cast<float*>(smem);  // [col][129]: reuses the drained stage ring
+    constexpr int pitch = 129;
+    if (warp < 8) {
+      for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
+        float v[32];
+        tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
+#pragma unroll
+        for (int i = 0; i < 32; ++i)
+          if (c0 + i < npad) P[(c0 + i) * pitch + trow] = v[i];
+      }
+    }
+    tc_fence_before();
     __syncthreads();
+    if (tid == 0) phase_mark(p, 3);
     const int v0 = blockIdx.y * 128;
     for (int c = tid; c < ncols; c += kThreads) {
       const RowDesc r = p.rows[col0 + c];
@@ -404,33 +468,70 @@ __global__ void __launch_bounds__(kThreads, 1)
         p.tok[r.slot] = y;
         p.res_tok[static_cast<size_t>(r.flags >> 8) * p.max_decode + r.b] = y;
       }
-      if (tid == 0) *p.done_ctas = 0;
+      __syncthreads();
+      if (tid == 0) {
+        *p.done_ctas = 0;
+        if (p.signal != nullptr) {  // completion signal (A12) fused into the last CTA
+          __threadfence_system();
+          atomicAdd_system(p.signal, 1ull);
+        }
+      }
     }
+    if (tid == 0) phase_mark(p, 4);
+    if (tid == 0) phase_mark(p, 5);
   } else {
     // ============================================================ split-K reduction + gates (A9)
-    cluster_sync();
-    if (tid == 0) phase_mark(p, 3);
+    // Each CTA owns a 1/S slice of the batch columns. After every CTA of the cluster finished
+    // its MMAs (barrier A), each CTA pushes its fp32 partial of every column to the owner's
+    // receive buffer R[src rank][owner column][tile row] with posted DSMEM stores; after
+    // barrier B each owner sums the S partials from its own smem in the fixed order
+    // s = 0..S-1 (deterministic, independent of the batch's other rows).
     const int S = p.S;
-    uint32_t peer[8];
-    for (int s = 0; s < S; ++s) peer[s] = mapa(smem_u32(P), s);
     const int cper = (ncols + S - 1) / S;
+    float* R = reinterpret_cast<float*>(smem);
+    cluster_sync();  // A: the cluster's MMAs are done -> every stage ring may be overwritten
+    if (tid == 0) phase_mark(p, 3);
+    if (warp < 8) {
+      uint32_t peer[kMaxS];
+#pragma unroll
+      for (int s = 0; s < kMaxS; ++s) peer[s] = mapa(smem_u32(R), s < S ? s : 0);
+      for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
+        float v[32];
+        tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
+#pragma unroll
+        for (int i = 0; i < 32; ++i) {
+          const int c = c0 + i;
+          if (c < ncols) {
+            const int owner = c / cper;
+            const int cl = c - owner * cper;
+            st_cluster_f32(peer[owner] + static_cast<uint32_t>(((rank * cper + cl) * 128 + trow) * 4), v[i]);
+          }
+        }
+      }
+    }
+    tc_fence_before();
+    cluster_sync();  // B: all partials delivered
+    if (tid == 0) phase_mark(p, 4);
     const int c_lo = static_cast<int>(rank) * cper;
-    const int c_hi = min(ncols, c_lo + cper);
+    const int my_cols = max(0, min(ncols, c_lo + cper) - c_lo);
     const int unit0 = blockIdx.y * U;
     const int prow0 = blockIdx.y * tile_rows;
     const size_t H = p.H;
     const size_t NS = p.n_slots;
     if (warp < 8) {
       const int cols_per_pass = kProducerThreads / U;
-      for (int c = c_lo + tid / U; c < c_hi; c += cols_per_pass) {
-        const int j = tid % U;
+      const int j = tid % U;
+      float bias[5];
+#pragma unroll
+      for (int g = 0; g < 5; ++g) bias[g] = g < G ? p.bias[prow0 + j * G + g] : 0.f;
+      for (int cl = tid / U; cl < my_cols; cl += cols_per_pass) {
         float z[5];
 #pragma unroll
-        for (int g = 0; g < 5; ++g) z[g] = 0.f;
-        const uint32_t off = static_cast<uint32_t>((c * pitch + j * G) * 4);
-        for (int s = 0; s < S; ++s) {  // fixed order -> deterministic, batch-invariant
+        for (int g = 0; g < 5; ++g) z[g] = bias[g];
+        for (int s = 0; s < S; ++s) {  // fixed order
+          const float* src = R + (s * cper + cl) * 128 + j * G;
           if (G == 4) {
-            const float4 v = ld_cluster_v4(peer[s] + off);
+            const float4 v = *reinterpret_cast<const float4*>(src);
             z[0] += v.x;
             z[1] += v.y;
             z[2] += v.z;
@@ -438,13 +539,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           } else {
 #pragma unroll
             for (int g = 0; g < 5; ++g)
-              if (g < G) z[g] += ld_cluster_f32(peer[s] + off + 4 * g);
+              if (g < G) z[g] += src[g];
           }
         }
-#pragma unroll
-        for (int g = 0; g < 5; ++g)
-          if (g < G) z[g] += p.bias[prow0 + j * G + g];
-        const RowDesc r = p.rows[col0 + c];
+        const RowDesc r = p.rows[col0 + c_lo + cl];
         const int u = unit0 + j;
         float hn, cn;
         if constexpr (EPI == EPI_LSTM) {
@@ -455,9 +553,9 @@ __global__ void __launch_bounds__(kThreads, 1)
           cn = sigm(z[0]) * tanhf(z[2]);
           hn = sigm(z[1]) * tanhf(cn);
         } else {
-          const float cl = p.c_pool[static_cast<size_t>(r.a) * H + u];
-          const float cr = p.c_pool[static_cast<size_t>(r.b) * H + u];
-          cn = sigm(z[0]) * tanhf(z[4]) + sigm(z[1]) * cl + sigm(z[2]) * cr;
+          const float cl_ = p.c_pool[static_cast<size_t>(r.a) * H + u];
+          const float cr_ = p.c_pool[static_cast<size_t>(r.b) * H + u];
+          cn = sigm(z[0]) * tanhf(z[4]) + sigm(z[1]) * cl_ + sigm(z[2]) * cr_;
           hn = sigm(z[3]) * tanhf(cn);
         }
         p.c_pool[r.slot * H + u] = cn;
@@ -470,12 +568,22 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
-    if (tid == 0) phase_mark(p, 4);
-    cluster_sync();  // peers may still read this CTA's partials until here
     if (tid == 0) phase_mark(p, 5);
+    if (p.signal != nullptr) {  // completion signal (A12) fused into the task's last CTA
+      __threadfence();
+      __syncthreads();
+      if (tid == 0) {
+        const unsigned total = gridDim.x * gridDim.y * gridDim.z;
+        if (atomicAdd(p.sig_ctas, 1u) == total - 1) {
+          *p.sig_ctas = 0;
+          __threadfence_system();
+          atomicAdd_system(p.signal, 1ull);
+        }
+      }
+    }
   }
 
-  if (warp == 8) {
+  if (warp == kMmaWarp) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256)
                  : "memory");
@@ -483,20 +591,18 @@ __global__ void __launch_bounds__(kThreads, 1)
 }
 
 template <int EPI>
-cudaError_t launch_impl(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t st) {
-  const int cols = a.b < kMaxCols ? a.b : kMaxCols;
-  const int npad = (cols + 15) & ~15;
-  const size_t smem = 1024 + kStages * (kWStageBytes + npad * 128) + 2 * kMaxCols * sizeof(void*) +
-                      (2 * kStages + 1) * 8 + 16;
+cudaError_t launch_impl(const StepArgs& a, cudaStream_t st) {
   static bool configured = false;
   if (!configured) {
+    const int max_smem = 1024 + kTailBytes + region_bytes(kMaxCols);
     cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         1024 + kStages * (kWStageBytes + kMaxCols * 128) +
-                                             2 * kMaxCols * (int)sizeof(void*) + (2 * kStages + 1) * 8 + 16);
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
     if (e != cudaSuccess) return e;
     configured = true;
   }
+  const int cols = a.b < kMaxCols ? a.b : kMaxCols;
+  const int npad = (cols + 15) & ~15;
+  const size_t smem = 1024 + kTailBytes + region_bytes(npad);
   const int S = EPI == EPI_PROJ ? 1 : a.S;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;
   cudaLaunchConfig_t cfg = {};
@@ -504,25 +610,27 @@ cudaError_t launch_impl(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t 
   cfg.blockDim = dim3(kThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = S;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI>, tmW, a);
+  cfg.numAttrs = 2;
+  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI>, a);
 }
 
 }  // namespace
 
-cudaError_t launch_cell_step_sm100(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t st) {
+cudaError_t launch_cell_step_sm100(const StepArgs& a, cudaStream_t st) {
   if (a.b <= 0) return cudaSuccess;
   switch (a.epi) {
-    case EPI_LSTM: return launch_impl<EPI_LSTM>(a, tmW, st);
-    case EPI_LEAF: return launch_impl<EPI_LEAF>(a, tmW, st);
-    case EPI_INTERNAL: return launch_impl<EPI_INTERNAL>(a, tmW, st);
-    case EPI_PROJ: return launch_impl<EPI_PROJ>(a, tmW, st);
+    case EPI_LSTM: return launch_impl<EPI_LSTM>(a, st);
+    case EPI_LEAF: return launch_impl<EPI_LEAF>(a, st);
+    case EPI_INTERNAL: return launch_impl<EPI_INTERNAL>(a, st);
+    case EPI_PROJ: return launch_impl<EPI_PROJ>(a, st);
   }
   return cudaErrorInvalidValue;
 }

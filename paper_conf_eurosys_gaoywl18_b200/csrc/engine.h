@@ -10,6 +10,7 @@
 #pragma once
 #include <stdint.h>
 
+#include <algorithm>
 #include <chrono>
 #include <deque>
 #include <string>
@@ -23,6 +24,53 @@ namespace bm {
 struct Engine;
 
 // ---------------------------------------------------------------- cell graph (A1, D1-D3)
+// Ready nodes of a subgraph, ascending (height, post-order index) [S18]. Chain / Seq2Seq
+// subgraphs hold at most one ready node, so small lists live inline (no heap, same cache line).
+struct ReadyList {
+  int n = 0;
+  int inl[2] = {0, 0};
+  std::vector<int> big;  // used once n would exceed the inline capacity (tree internal)
+  int size() const { return n; }
+  int operator[](int i) const { return big.empty() ? inl[i] : big[i]; }
+  void clear() {
+    n = 0;
+    big.clear();
+  }
+  void assign1(int v) {
+    clear();
+    inl[0] = v;
+    n = 1;
+  }
+  void insert_at(int pos, int v) {
+    if (big.empty() && n < 2) {
+      for (int i = n; i > pos; --i) inl[i] = inl[i - 1];
+      inl[pos] = v;
+      ++n;
+      return;
+    }
+    if (big.empty()) big.assign(inl, inl + n);
+    big.insert(big.begin() + pos, v);
+    ++n;
+  }
+  void erase_value(int v) {
+    if (big.empty()) {
+      int i = 0;
+      while (i < n && inl[i] != v) ++i;
+      for (; i + 1 < n; ++i) inl[i] = inl[i + 1];
+      --n;
+      return;
+    }
+    big.erase(std::find(big.begin(), big.end(), v));
+    --n;
+    if (n == 0) big.clear();
+  }
+  bool contains(int v) const {
+    for (int i = 0; i < n; ++i)
+      if ((*this)[i] == v) return true;
+    return false;
+  }
+};
+
 struct Subgraph {
   int req = -1;            // request table index
   int sid = 0;             // subgraph id within the request
@@ -32,32 +80,40 @@ struct Subgraph {
   int n_completed = 0;
   int pinned = -1;         // worker id or -1 (Alg. 1 line 21, L381)
   int inflight = 0;        // tasks in flight holding nodes of this subgraph
-  std::vector<int> ready;  // ready, unsubmitted nodes, ascending (height, post-order index)
   // intrusive FIFO links of the cell type's subgraph queue (D3)
   int q_prev_req = -1, q_prev_sid = -1, q_next_req = -1, q_next_sid = -1;
   bool queued = false;
+  ReadyList ready;
 };
 
+// Hot fields first: the scheduler touches a request several times per scheduled node.
 struct Request {
-  bool used = false;
-  bool done = false;
-  uint64_t id = 0;          // admission index
-  uint64_t tag = 0;
   int kind = 0;
   int cell0 = 0, cell1 = 0;
   int n_nodes = 0;          // chain: L; seq2seq: S + T; tree: n
   int enc_len = 0;          // seq2seq: S
   int n_completed = 0;
+  int slot = -1;            // chain / seq2seq
   int leaves_left = 0;
   int internal_sid = -1;
+  bool used = false;
+  bool done = false;
   bool started = false;     // slots taken
-  int slot = -1;            // chain / seq2seq
+  uint64_t id = 0;          // admission index
+  uint64_t tag = 0;
   double t_arrival = 0, t_first = -1, t_done = -1;
+  Subgraph sg2[2];          // chain: [0]; seq2seq: encoder [0], decoder [1]
   std::vector<int32_t> tokens;      // chain/seq2seq: source tokens; tree: per node
+  // trees only
+  std::vector<Subgraph> sgv;        // leaf subgraphs then the internal subgraph
   std::vector<int32_t> left, right, parent, height, node_slot;
   std::vector<uint8_t> submitted;
-  std::vector<Subgraph> sg;
-  std::vector<int> node_sid;        // trees: subgraph of each node
+  std::vector<int> node_sid;        // subgraph of each node
+  Subgraph& sg(int sid) { return kind == BM_REQ_TREE ? sgv[sid] : sg2[sid]; }
+  const Subgraph& sg(int sid) const { return kind == BM_REQ_TREE ? sgv[sid] : sg2[sid]; }
+  int sid_of(int node) const {
+    return kind == BM_REQ_TREE ? node_sid[node] : (kind == BM_REQ_SEQ2SEQ && node >= enc_len ? 1 : 0);
+  }
 };
 
 struct Cell {
@@ -66,11 +122,9 @@ struct Cell {
   // device weights (per layer for LSTM stacks)
   std::vector<void*> W;
   std::vector<float*> bias;
-  std::vector<CUtensorMap> tm;
   void* E = nullptr;
   void* W_out = nullptr;
   float* b_out = nullptr;
-  CUtensorMap tm_out{};
   // scheduler state of this cell type
   int q_head_req = -1, q_head_sid = -1, q_tail_req = -1, q_tail_sid = -1;
   int64_t ready_nodes = 0;   // NumReadyNodes (S16)
@@ -91,6 +145,7 @@ struct Task {
   int ring_off = 0;          // first row in the descriptor ring
   int b = 0;
   std::vector<TaskRow> rows;
+  std::vector<RowDesc> desc; // device row descriptors, built at submission (A3)
   int ev_first = -1, ev_count = 0;  // timed launches (time_kernels)
 };
 
@@ -132,6 +187,7 @@ struct Engine {
   int logits_vocab = 0;
   unsigned long long* amax = nullptr;
   unsigned int* done_ctas = nullptr;
+  unsigned int* sig_ctas = nullptr;  // CTA counter of the fused completion signal
   RowDesc* ring_dev = nullptr;
   RowDesc* ring_host = nullptr;    // pinned staging
   int ring_rows = 0;
@@ -141,6 +197,9 @@ struct Engine {
   unsigned long long* signal_dev = nullptr;
   RowDesc* direct_rows = nullptr;  // bm_cell_step rows (device)
   unsigned long long* phase_dev = nullptr;  // BM_PHASE_DUMP diagnostics
+  RowDesc* direct_host = nullptr;  // pinned staging of bm_cell_step rows (double buffered)
+  cudaEvent_t direct_ev[2] = {nullptr, nullptr};
+  int direct_flip = 0;
   std::vector<TimedLaunch> ev_pool;
   int ev_head = 0;
 

@@ -44,7 +44,7 @@ struct StepArgs {
   void* h_pool;         // pool h of this layer ([2][n_slots][H])
   float* c_pool;        // pool c of this layer ([n_slots][H])
   int* tok;             // feed tokens [n_slots]
-  const void* W;        // packed weights [rows][K] (SIMT path; the bf16 path uses the TMA map)
+  const void* W;        // fp32 path: packed [rows][K]; bf16 path: stage tiles (launch_pack_tiles)
   const float* bias;    // packed bias [rows]
   int W_rows;           // G * H (or V for the projection)
   float* res_h;         // result rows [max_requests][res_layers][H]
@@ -57,16 +57,24 @@ struct StepArgs {
   int max_decode;
   float* logits;              // debug [max_requests][max_decode][V] or null
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer at phase boundaries, or null
+  int max_stages;             // experiments (BM_MAX_STAGES): cap on pipeline stages, 0 = default
+  // launch path
+  unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
+  unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)
+  int pdl;                    // launch with programmatic dependent launch (overlap setup)
 };
 
-// bf16 / tcgen05 path (cell_step_sm100.cu). tmW: TMA map of the packed bf16 weights.
-cudaError_t launch_cell_step_sm100(const StepArgs& a, const CUtensorMap& tmW, cudaStream_t st);
+// bf16 / tcgen05 path (cell_step_sm100.cu). a.W: weights in the stage-tile layout
+// (launch_pack_tiles): [tile][K/64][tile_rows][64] bf16, 128B-swizzled rows.
+cudaError_t launch_cell_step_sm100(const StepArgs& a, cudaStream_t st);
 // fp32 / SIMT path (cell_step_simt.cu)
 cudaError_t launch_cell_step_simt(const StepArgs& a, cudaStream_t st);
 
 // Weight preparation (load time): fp32 paper layout -> packed, gate-interleaved, bf16 or fp32.
 cudaError_t launch_pack_rows(const float* src, void* dst, float* bias_dst, const float* bias_src,
                              int G, int H, int K, int bf16, cudaStream_t st);
+cudaError_t launch_pack_tiles(const float* src, void* dst, int G, int H, int K, int tile_rows,
+                              int n_rows, cudaStream_t st);
 cudaError_t launch_convert(const float* src, void* dst, size_t n, int bf16, cudaStream_t st);
 // Completion signal (A12): bump a host-mapped counter after everything before it in stream.
 cudaError_t launch_signal(unsigned long long* counter, cudaStream_t st);

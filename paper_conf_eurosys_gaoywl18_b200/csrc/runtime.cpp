@@ -35,36 +35,6 @@ namespace {
     }                                 \
   } while (0)
 
-typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
-                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
-                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
-                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-EncodeTiledFn encode_fn() {
-  static EncodeTiledFn fn = nullptr;
-  if (fn == nullptr) {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<EncodeTiledFn>(p);
-  }
-  return fn;
-}
-
-// TMA map of a packed bf16 matrix [rows][K], box = 64 K-elements x box_rows, 128B swizzle.
-bool make_tmap(CUtensorMap* m, const void* base, int rows, int K, int box_rows) {
-  EncodeTiledFn fn = encode_fn();
-  if (fn == nullptr) return false;
-  cuuint64_t dims[2] = {static_cast<cuuint64_t>(K), static_cast<cuuint64_t>(rows)};
-  cuuint64_t strides[1] = {static_cast<cuuint64_t>(K) * 2};
-  cuuint32_t box[2] = {64, static_cast<cuuint32_t>(box_rows)};
-  cuuint32_t es[2] = {1, 1};
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
-            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
-
 template <class T>
 cudaError_t dalloc(T** p, size_t n) {
   return cudaMalloc(reinterpret_cast<void**>(p), n * sizeof(T));
@@ -94,7 +64,7 @@ void algo_cost(const Engine& e, const Cell& c, int b, bool proj, double* bytes, 
 
 // ---------------------------------------------------------------- launching tasks
 static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, int b, int layer,
-                                 bool proj, int* ev_out) {
+                                 bool proj, int* ev_out, unsigned long long* signal) {
   StepArgs a{};
   a.epi = proj ? EPI_PROJ : c.epi;
   a.G = proj ? 1 : c.G;
@@ -132,6 +102,11 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
   a.max_decode = e.cfg.max_decode_len;
   a.logits = (proj && e.logits != nullptr) ? e.logits : nullptr;
   a.phase = e.phase_dev;
+  static const int max_stages = getenv("BM_MAX_STAGES") ? atoi(getenv("BM_MAX_STAGES")) : 0;
+  a.max_stages = max_stages;
+  a.signal = signal;
+  a.sig_ctas = e.sig_ctas;
+  a.pdl = 1;
   TimedLaunch* tl = nullptr;
   if (e.cfg.time_kernels && !e.ev_pool.empty()) {
     const int i = e.ev_head;
@@ -142,66 +117,48 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
     if (ev_out) *ev_out = i;
   }
   cudaError_t err;
-  if (e.cfg.precision == BM_PREC_BF16) err = launch_cell_step_sm100(a, proj ? c.tm_out : c.tm[layer], e.stream);
-  else err = launch_cell_step_simt(a, e.stream);
+  if (e.cfg.precision == BM_PREC_BF16) {
+    err = launch_cell_step_sm100(a, e.stream);
+  } else {
+    a.pdl = 0;  // the SIMT kernels do not use griddepcontrol
+    err = launch_cell_step_simt(a, e.stream);
+  }
   CK(err);
   if (tl) CK(cudaEventRecord(tl->end, e.stream));
   e.stats.kernel_launches += 1;
   return BM_OK;
 }
 
-static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, int b, Task* t) {
+// All kernels of one task in order on the engine stream (§5). With `signal`, the task's
+// completion is signalled: fused into the last kernel's last CTA on the tcgen05 path (A12),
+// or by the signal kernel on the fp32 path.
+static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, int b, Task* t,
+                             unsigned long long* signal) {
   const bool lstm = c.epi == EPI_LSTM;
+  const bool proj = c.d.kind == BM_CELL_LSTM_PROJ;
+  const bool fused = e.cfg.precision == BM_PREC_BF16;
   const int L = lstm ? c.d.layers : 1;
   for (int l = 0; l < L; ++l) {
     int ev = -1;
-    bm_status s = launch_one_step(e, c, rows_dev, b, l, false, &ev);
+    const bool last = l == L - 1 && !proj;
+    bm_status s = launch_one_step(e, c, rows_dev, b, l, false, &ev, (last && fused) ? signal : nullptr);
     if (s != BM_OK) return s;
     if (t && ev >= 0) {
       if (t->ev_first < 0) t->ev_first = ev;
       t->ev_count += 1;
     }
   }
-  if (c.d.kind == BM_CELL_LSTM_PROJ) {
+  if (proj) {
     int ev = -1;
-    bm_status s = launch_one_step(e, c, rows_dev, b, 0, true, &ev);
+    bm_status s = launch_one_step(e, c, rows_dev, b, 0, true, &ev, fused ? signal : nullptr);
     if (s != BM_OK) return s;
     if (t && ev >= 0) t->ev_count += 1;
   }
-  return BM_OK;
-}
-
-// Row descriptor of a scheduled node (A3): what the kernels need to gather and scatter.
-static RowDesc make_row(const Engine& e, const Cell& c, const TaskRow& tr) {
-  const Request& r = e.reqs[tr.req];
-  RowDesc d{};
-  d.slot = tr.slot;
-  int flags = 0;
-  const int res = tr.req;  // result row = request table index
-  if (r.kind == BM_REQ_TREE) {
-    if (r.left[tr.node] < 0) {
-      d.a = r.tokens[tr.node];
-    } else {
-      d.a = r.node_slot[r.left[tr.node]];
-      d.b = r.node_slot[r.right[tr.node]];
-    }
-    if (tr.node == r.n_nodes - 1) flags |= ROW_LAST;
-  } else {
-    const int step = tr.node;  // global step (encoder steps then decoder steps)
-    if (step == 0) flags |= ROW_FIRST;
-    if (step & 1) flags |= ROW_PARITY;
-    if (r.kind == BM_REQ_CHAIN || step < r.enc_len) {
-      d.a = r.tokens[step];
-    } else {
-      const int s = step - r.enc_len;
-      d.a = s == 0 ? 1 /* <go> */ : -1 /* feed previous: tok[slot] on device */;
-      d.b = s;
-    }
-    if (step == r.n_nodes - 1) flags |= ROW_LAST;
+  if (signal != nullptr && !fused) {
+    CK(launch_signal(signal, e.stream));
+    e.stats.kernel_launches += 1;
   }
-  (void)c;
-  d.flags = flags | (res << 8);
-  return d;
+  return BM_OK;
 }
 
 bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
@@ -218,14 +175,16 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
       t.finish = start + 1.0;
       e.last_finish = t.finish;
     }
-    bm_task_record rec;
-    rec.task = static_cast<int>(t.seq);
-    rec.cell = t.ct;
-    rec.tick = t.tick;
-    rec.first_row = static_cast<int>(e.log_rows.size());
-    rec.n_rows = t.b;
-    e.log_tasks.push_back(rec);
-    for (const TaskRow& tr : t.rows) e.log_rows.push_back({e.reqs[tr.req].id, tr.node, tr.slot});
+    if (e.cfg.record_log) {
+      bm_task_record rec;
+      rec.task = static_cast<int>(t.seq);
+      rec.cell = t.ct;
+      rec.tick = t.tick;
+      rec.first_row = static_cast<int>(e.log_rows.size());
+      rec.n_rows = t.b;
+      e.log_tasks.push_back(rec);
+      for (const TaskRow& tr : t.rows) e.log_rows.push_back({e.reqs[tr.req].id, tr.node, tr.slot});
+    }
   }
   if (!e.device()) return BM_OK;
   // ring placement: one contiguous region for all tasks of this Schedule call
@@ -235,18 +194,15 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
   int off = base;
   for (Task& t : tasks) {
     t.ring_off = off;
-    Cell& c = e.cells[t.ct];
-    for (int i = 0; i < t.b; ++i) e.ring_host[off + i] = make_row(e, c, t.rows[i]);
+    memcpy(e.ring_host + off, t.desc.data(), sizeof(RowDesc) * t.b);
     off += t.b;
   }
   e.ring_head = off;
   CK(cudaMemcpyAsync(e.ring_dev + base, e.ring_host + base, sizeof(RowDesc) * total,
                      cudaMemcpyHostToDevice, e.stream));
   for (Task& t : tasks) {
-    bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, t.b, &t);
+    bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, t.b, &t, e.signal_dev);
     if (s != BM_OK) return s;
-    CK(launch_signal(e.signal_dev, e.stream));
-    e.stats.kernel_launches += 1;
   }
   return BM_OK;
 }
@@ -368,6 +324,7 @@ void bm_config_default(bm_config* c) {
   c->keep_results = 0;
   c->record_logits = 0;
   c->time_kernels = 0;
+  c->record_log = 1;
 }
 
 static void free_device(Engine& e) {
@@ -388,9 +345,13 @@ static void free_device(Engine& e) {
   cudaFree(e.logits);
   cudaFree(e.amax);
   cudaFree(e.done_ctas);
+  cudaFree(e.sig_ctas);
   cudaFree(e.ring_dev);
   cudaFree(e.direct_rows);
   cudaFree(e.phase_dev);
+  if (e.direct_host) cudaFreeHost(e.direct_host);
+  for (cudaEvent_t ev : e.direct_ev)
+    if (ev) cudaEventDestroy(ev);
   if (e.ring_host) cudaFreeHost(e.ring_host);
   if (e.signal_host) cudaFreeHost(e.signal_host);
   for (TimedLaunch& t : e.ev_pool) {
@@ -436,7 +397,10 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
               dalloc(&E.res_h, R * L * H) == cudaSuccess && dalloc(&E.res_c, R * L * H) == cudaSuccess &&
               dalloc(&E.res_tok, R * static_cast<size_t>(c.max_decode_len)) == cudaSuccess &&
               dalloc(&E.amax, 512) == cudaSuccess && dalloc(&E.done_ctas, 1) == cudaSuccess &&
-              dalloc(&E.direct_rows, 4096) == cudaSuccess;
+              dalloc(&E.sig_ctas, 1) == cudaSuccess &&
+              dalloc(&E.direct_rows, 2 * 4096) == cudaSuccess &&
+              cudaEventCreateWithFlags(&E.direct_ev[0], cudaEventDisableTiming) == cudaSuccess &&
+              cudaEventCreateWithFlags(&E.direct_ev[1], cudaEventDisableTiming) == cudaSuccess;
     if (!ok) return fail(BM_E_NOMEM);
     E.ring_rows = std::max(64, c.max_tasks_to_submit + c.schedule_when_outstanding_leq + 2) * 512 * 2;
     if (dalloc(&E.ring_dev, E.ring_rows) != cudaSuccess) return fail(BM_E_NOMEM);
@@ -454,6 +418,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
         cudaMemsetAsync(E.tok, 0, S * 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.amax, 0, 512 * 8, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.done_ctas, 0, 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.sig_ctas, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.res_tok, 0, R * c.max_decode_len * 4, E.stream) != cudaSuccess)
       return fail(BM_E_CUDA);
     if (c.time_kernels) {
@@ -534,14 +499,11 @@ bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w,
       CK(cudaMemcpyAsync(tmp, w->W[l], rows * K * 4, cudaMemcpyHostToDevice, e.stream));
       CK(cudaMemcpyAsync(tmpb, w->b[l], rows * 4, cudaMemcpyHostToDevice, e.stream));
       CK(launch_pack_rows(tmp, Wp, bp, tmpb, c.G, H, K, bf ? 1 : 0, e.stream));
+      if (bf)  // the tcgen05 kernel streams pre-swizzled stage tiles (overwrites the plain pack)
+        CK(launch_pack_tiles(tmp, Wp, c.G, H, K, c.G * c.U, static_cast<int>(rows), e.stream));
       CK(cudaStreamSynchronize(e.stream));
       c.W.push_back(Wp);
       c.bias.push_back(bp);
-      if (bf) {
-        CUtensorMap m;
-        if (!make_tmap(&m, Wp, static_cast<int>(rows), K, c.G * c.U)) return BM_E_CUDA;
-        c.tm.push_back(m);
-      }
     }
     if (w->E != nullptr && d->kind != BM_CELL_TREE_INTERNAL) {
       const size_t n = static_cast<size_t>(d->vocab) * H;
@@ -555,10 +517,10 @@ bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w,
       CK(cudaMalloc(&c.W_out, n * el));
       CK(dalloc(&c.b_out, d->vocab));
       CK(cudaMemcpyAsync(tmp, w->W_out, n * 4, cudaMemcpyHostToDevice, e.stream));
-      CK(launch_convert(tmp, c.W_out, n, bf ? 1 : 0, e.stream));
+      if (bf) CK(launch_pack_tiles(tmp, c.W_out, 1, H, H, 128, d->vocab, e.stream));
+      else CK(launch_convert(tmp, c.W_out, n, 0, e.stream));
       CK(cudaMemcpyAsync(c.b_out, w->b_out, d->vocab * 4, cudaMemcpyHostToDevice, e.stream));
       CK(cudaStreamSynchronize(e.stream));
-      if (bf && !make_tmap(&c.tm_out, c.W_out, d->vocab, H, 128)) return BM_E_CUDA;
       if (e.cfg.record_logits) {
         if (e.logits == nullptr) {
           CK(dalloc(&e.logits, static_cast<size_t>(e.cfg.max_requests) * e.cfg.max_decode_len * d->vocab));
@@ -838,12 +800,20 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
     if (rows[i].slot < 0 || rows[i].slot >= e.cfg.max_slots) return BM_E_INVAL;
     if ((rows[i].flags >> 8) >= e.cfg.max_requests) return BM_E_INVAL;
   }
-  CK(cudaMemcpyAsync(e.direct_rows, rows, sizeof(RowDesc) * b, cudaMemcpyHostToDevice, e.stream));
+  // stage through pinned memory so the copy is truly asynchronous (back-to-back direct steps)
+  if (e.direct_host == nullptr)
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&e.direct_host), sizeof(RowDesc) * 4096 * 2, cudaHostAllocDefault));
+  RowDesc* stage = e.direct_host + (e.direct_flip ^= 1) * 4096;
+  if (async) CK(cudaEventSynchronize(e.direct_ev[e.direct_flip]));
+  memcpy(stage, rows, sizeof(RowDesc) * b);
+  CK(cudaMemcpyAsync(e.direct_rows + e.direct_flip * 4096, stage, sizeof(RowDesc) * b, cudaMemcpyHostToDevice, e.stream));
+  CK(cudaEventRecord(e.direct_ev[e.direct_flip], e.stream));
+  RowDesc* rows_dev = e.direct_rows + e.direct_flip * 4096;
   // diagnostics: BM_PHASE_DUMP=<file> records per-CTA phase timestamps of every direct step
   static const char* dump = getenv("BM_PHASE_DUMP");
   if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 8 * 4096));
   if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 8 * 4096, e.stream));
-  bm_status s = launch_cell(e, c, e.direct_rows, b, nullptr);
+  bm_status s = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
   if (s != BM_OK) return s;
   if (!async || e.phase_dev) CK(cudaStreamSynchronize(e.stream));
   if (e.phase_dev) {

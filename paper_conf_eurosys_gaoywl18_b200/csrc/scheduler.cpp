@@ -22,7 +22,7 @@
 namespace bm {
 namespace {
 
-inline Subgraph& SG(Engine& e, int req, int sid) { return e.reqs[req].sg[sid]; }
+inline Subgraph& SG(Engine& e, int req, int sid) { return e.reqs[req].sg(sid); }
 
 void enqueue(Engine& e, int req, int sid) {  // append to the cell type's FIFO [S18]
   Subgraph& g = SG(e, req, sid);
@@ -70,12 +70,14 @@ void dequeue(Engine& e, int req, int sid) {
 // insert node v into the subgraph's ready list keeping (height, index) order [S18]
 void make_ready(Engine& e, int req, int sid, int v) {
   Request& r = e.reqs[req];
-  Subgraph& g = r.sg[sid];
-  const int hv = r.kind == BM_REQ_TREE ? r.height[v] : v;
-  auto key = [&](int u) { return r.kind == BM_REQ_TREE ? std::make_pair(r.height[u], u) : std::make_pair(u, u); };
-  auto it = std::upper_bound(g.ready.begin(), g.ready.end(), std::make_pair(hv, v),
-                             [&](const std::pair<int, int>& k, int u) { return k < key(u); });
-  g.ready.insert(it, v);
+  Subgraph& g = r.sg(sid);
+  int pos = g.ready.size();
+  if (r.kind == BM_REQ_TREE) {
+    const std::pair<int, int> kv(r.height[v], v);
+    pos = 0;
+    while (pos < g.ready.size() && std::make_pair(r.height[g.ready[pos]], g.ready[pos]) < kv) ++pos;
+  }
+  g.ready.insert_at(pos, v);
   if (g.queued) e.cells[g.ct].ready_nodes += 1;
 }
 
@@ -104,24 +106,23 @@ bool has_ready(const Engine& e) {
 // ---------------------------------------------------------------- admission (A1)
 bm_status admit_request(Engine& e, int ri) {
   Request& r = e.reqs[ri];
-  r.sg.clear();
   r.n_completed = 0;
   r.started = false;
   r.slot = -1;
   r.t_first = -1;
   r.t_done = -1;
-  r.submitted.assign(r.n_nodes, 0);
   if (r.kind == BM_REQ_CHAIN || r.kind == BM_REQ_SEQ2SEQ) {
     const int S = r.kind == BM_REQ_CHAIN ? r.n_nodes : r.enc_len;
-    r.sg.resize(r.kind == BM_REQ_CHAIN ? 1 : 2);
-    Subgraph& enc = r.sg[0];
+    r.sg2[0] = Subgraph();
+    r.sg2[1] = Subgraph();
+    Subgraph& enc = r.sg2[0];
     enc.req = ri;
     enc.sid = 0;
     enc.ct = r.cell0;
     enc.n_nodes = S;
-    enc.ready.assign(1, 0);
+    enc.ready.assign1(0);
     if (r.kind == BM_REQ_SEQ2SEQ) {
-      Subgraph& dec = r.sg[1];
+      Subgraph& dec = r.sg2[1];
       dec.req = ri;
       dec.sid = 1;
       dec.ct = r.cell1;
@@ -130,6 +131,7 @@ bm_status admit_request(Engine& e, int ri) {
     enqueue(e, ri, 0);
   } else {
     const int n = r.n_nodes;
+    r.submitted.assign(n, 0);
     r.parent.assign(n, -1);
     r.height.assign(n, 0);
     r.node_slot.assign(n, -1);
@@ -145,22 +147,22 @@ bm_status admit_request(Engine& e, int ri) {
       }
     }
     r.leaves_left = n_leaves;
-    r.sg.resize(n_leaves + (n > n_leaves ? 1 : 0));
+    r.sgv.assign(n_leaves + (n > n_leaves ? 1 : 0), Subgraph());
     int sid = 0;
     for (int v = 0; v < n; ++v) {
       if (r.left[v] >= 0) continue;
-      Subgraph& g = r.sg[sid];
+      Subgraph& g = r.sgv[sid];
       g.req = ri;
       g.sid = sid;
       g.ct = r.cell0;
       g.n_nodes = 1;
-      g.ready.assign(1, v);
+      g.ready.assign1(v);
       r.node_sid[v] = sid;
       ++sid;
     }
     r.internal_sid = -1;
     if (n > n_leaves) {
-      Subgraph& g = r.sg[sid];
+      Subgraph& g = r.sgv[sid];
       g.req = ri;
       g.sid = sid;
       g.ct = r.cell1;
@@ -195,7 +197,8 @@ void form_batched_task(Engine& e, int ct, int worker, std::vector<Cand>& batch) 
     const int nreq = g.q_next_req, nsid = g.q_next_sid;
     if (g.pinned < 0 || g.pinned == worker) {                     // line 27
       Request& r = e.reqs[req];
-      for (int v : g.ready) {                                     // line 28
+      for (int i = 0; i < g.ready.size(); ++i) {                  // line 28
+        const int v = g.ready[i];
         int need = 0;
         if (!r.started && last_new_req != req) need = slots_needed(r);
         if (need > free) break;
@@ -220,10 +223,39 @@ void release_successor(Engine& e, int req, int sid, int v) {  // UpdateNodesDepe
     const int p = r.parent[v];
     if (p >= 0 && r.node_sid[p] == sid && !r.submitted[p] && r.submitted[r.left[p]] &&
         r.submitted[r.right[p]]) {
-      Subgraph& g = r.sg[sid];
-      if (std::find(g.ready.begin(), g.ready.end(), p) == g.ready.end()) make_ready(e, req, sid, p);
+      if (!r.sg(sid).ready.contains(p)) make_ready(e, req, sid, p);
     }
   }
+}
+
+// Device row descriptor of a scheduled node (A3): what the kernels need to gather and scatter.
+RowDesc describe_row(const Request& r, int ri, int node, int slot) {
+  RowDesc d{};
+  d.slot = slot;
+  int flags = 0;
+  if (r.kind == BM_REQ_TREE) {
+    if (r.left[node] < 0) {
+      d.a = r.tokens[node];
+    } else {
+      d.a = r.node_slot[r.left[node]];
+      d.b = r.node_slot[r.right[node]];
+    }
+    if (node == r.n_nodes - 1) flags |= ROW_LAST;
+  } else {
+    const int step = node;  // global step (encoder steps then decoder steps)
+    if (step == 0) flags |= ROW_FIRST;
+    if (step & 1) flags |= ROW_PARITY;
+    if (r.kind == BM_REQ_CHAIN || step < r.enc_len) {
+      d.a = r.tokens[step];
+    } else {
+      const int s = step - r.enc_len;
+      d.a = s == 0 ? 1 /* <go> */ : -1 /* feed previous: tok[slot] on device */;
+      d.b = s;
+    }
+    if (step == r.n_nodes - 1) flags |= ROW_LAST;
+  }
+  d.flags = flags | (ri << 8);  // result row = request table index
+  return d;
 }
 
 Task submit(Engine& e, int ct, int worker, const std::vector<Cand>& batch) {
@@ -231,6 +263,7 @@ Task submit(Engine& e, int ct, int worker, const std::vector<Cand>& batch) {
   t.ct = ct;
   t.tick = e.now;
   t.rows.reserve(batch.size());
+  t.desc.reserve(batch.size());
   Cell& c = e.cells[ct];
   for (const Cand& x : batch) {
     Request& r = e.reqs[x.req];
@@ -245,11 +278,12 @@ Task submit(Engine& e, int ct, int worker, const std::vector<Cand>& batch) {
     if (r.t_first < 0) r.t_first = e.now;
     const int slot = r.kind == BM_REQ_TREE ? r.node_slot[x.node] : r.slot;
     t.rows.push_back({x.req, x.node, slot});
-    Subgraph& g = r.sg[x.sid];
-    g.ready.erase(std::find(g.ready.begin(), g.ready.end(), x.node));
+    Subgraph& g = r.sg(x.sid);
+    g.ready.erase_value(x.node);
     if (g.queued) c.ready_nodes -= 1;
     g.n_submitted += 1;
-    r.submitted[x.node] = 1;
+    if (r.kind == BM_REQ_TREE) r.submitted[x.node] = 1;
+    t.desc.push_back(describe_row(r, x.req, x.node, slot));
   }
   c.running_tasks += 1;
   for (const Cand& x : batch) release_successor(e, x.req, x.sid, x.node);   // line 18
@@ -320,15 +354,12 @@ void retire_task(Engine& e, Task& t) {
   for (size_t i = 0; i < t.rows.size(); ++i) {
     const TaskRow& row = t.rows[i];
     Request& r = e.reqs[row.req];
-    const int sid = r.kind == BM_REQ_TREE ? r.node_sid[row.node]
-                                           : (r.kind == BM_REQ_SEQ2SEQ && row.node >= r.enc_len ? 1 : 0);
-    Subgraph& g = r.sg[sid];
+    const int sid = r.sid_of(row.node);
+    Subgraph& g = r.sg(sid);
     bool seen = false;  // rows of one subgraph are contiguous (see submit)
     if (i > 0 && t.rows[i - 1].req == row.req) {
       const TaskRow& o = t.rows[i - 1];
-      const int osid = r.kind == BM_REQ_TREE ? r.node_sid[o.node]
-                                             : (r.kind == BM_REQ_SEQ2SEQ && o.node >= r.enc_len ? 1 : 0);
-      seen = osid == sid;
+      seen = r.sid_of(o.node) == sid;
     }
     if (!seen) {
       g.inflight -= 1;
@@ -337,12 +368,12 @@ void retire_task(Engine& e, Task& t) {
     g.n_completed += 1;
     r.n_completed += 1;
     if (g.n_completed == g.n_nodes) {       // subgraph done: inter-subgraph deps [S20]
-      if (r.kind == BM_REQ_SEQ2SEQ && sid == 0 && r.sg[1].n_nodes > 0) {
-        r.sg[1].ready.assign(1, r.enc_len);
+      if (r.kind == BM_REQ_SEQ2SEQ && sid == 0 && r.sg2[1].n_nodes > 0) {
+        r.sg2[1].ready.assign1(r.enc_len);
         enqueue(e, row.req, 1);
       } else if (r.kind == BM_REQ_TREE && r.left[row.node] < 0) {
         if (--r.leaves_left == 0 && r.internal_sid >= 0) {
-          Subgraph& is = r.sg[r.internal_sid];
+          Subgraph& is = r.sgv[r.internal_sid];
           is.ready.clear();
           enqueue(e, row.req, r.internal_sid);
           for (int v = 0; v < r.n_nodes; ++v)

@@ -13,7 +13,7 @@ for line in open(sys.argv[1]):
         steps.append(cur)
     else:
         v = [int(x) for x in line.split()]
-        cur["rows"].append(v[1:7])
+        cur["rows"].append(v[1:9])
 for st in steps[-3:]:
     a = np.array(st["rows"], dtype=np.float64)
     t0 = a[:, 0].min()
@@ -23,3 +23,6 @@ for st in steps[-3:]:
     for k in range(1, 6):
         d = (a[:, k] - a[:, k - 1]) / 1e3
         print("  %-8s us: min %.2f med %.2f max %.2f" % (names[k], d.min(), np.median(d), d.max()))
+    for k, nm in ((6, "first stage at MMA (from setup)"), (7, "last stage at MMA (from setup)")):
+        d = (a[:, k] - a[:, 1]) / 1e3
+        print("  %-32s us: min %.2f med %.2f max %.2f" % (nm, d.min(), np.median(d), d.max()))
