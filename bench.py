@@ -34,7 +34,12 @@ import sys
 import threading
 import time
 
-import numpy as np
+# the CPU oracle baseline forks one process per core: pin BLAS to one thread per process
+# BEFORE numpy is imported (an inherited multi-threaded BLAS would oversubscribe the cores)
+for _v in ("OMP_NUM_THREADS", "OPENBLAS_NUM_THREADS", "MKL_NUM_THREADS"):
+    os.environ.setdefault(_v, "1")
+
+import numpy as np  # noqa: E402
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
@@ -54,7 +59,7 @@ def parse():
     p.add_argument("--reqs", type=int, default=0, help="requests per step (0 = per-workload default)")
     p.add_argument("--p90-ms", type=float, default=12.0)
     p.add_argument("--rate", type=float, default=0.0, help="skip the sweep, use this offered rate")
-    p.add_argument("--lookahead", type=int, default=2,
+    p.add_argument("--lookahead", type=int, default=8,
                    help="schedule when <= k tasks are outstanding (0 = the paper's idle-only)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
@@ -403,9 +408,14 @@ def main():
     hbm = peaks.get("hbm_gbs", 6650.0)
     achieved = st["timed_bytes"] / (st["timed_ms"] / 1e3) / 1e9 if st["timed_ms"] > 0 else 0.0
     tflops = st["timed_flops"] / (st["timed_ms"] / 1e3) / 1e12 if st["timed_ms"] > 0 else 0.0
+    span_gbs = st["timed_bytes"] / (st["span_ms"] / 1e3) / 1e9 if st["span_ms"] > 0 else 0.0
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
             "traffic": None, "kernel": "cell_step_sm100_kernel", "launches": st["timed_launches"],
             "avg_launch_us": st["timed_ms"] * 1e3 / max(1, st["timed_launches"]),
+            "device_span": {"avg_launch_us": st["span_ms"] * 1e3 / max(1, st["timed_launches"]),
+                            "achieved": span_gbs, "frac": span_gbs / hbm,
+                            "note": "first-CTA-start to last-CTA-end per launch (%globaltimer); "
+                                    "excludes host launch latency the CUDA-event bracket includes"},
             "avg_rows_per_task": st["rows"] / max(1, st["tasks"]), "tensor_tflops": tflops,
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)" if peaks else "fallback 6.65 TB/s"}
     cpu = None

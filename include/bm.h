@@ -251,6 +251,8 @@ typedef struct {
   double timed_flops;        /* sum of their algorithmic flops                           */
   double sched_ns;           /* host time spent in Schedule/Batch                        */
   uint64_t schedule_calls;
+  double span_ms;            /* same launches, device-side span (first CTA start .. last  */
+                             /* CTA end, %globaltimer): excludes host launch latency      */
 } bm_stats;
 
 bm_status bm_get_stats(bm_engine* e, bm_stats* out);

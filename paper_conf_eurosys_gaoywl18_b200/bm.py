@@ -81,7 +81,7 @@ class Stats(C.Structure):
     _fields_ = [("tasks", C.c_uint64), ("rows", C.c_uint64), ("kernel_launches", C.c_uint64),
                 ("timed_launches", C.c_uint64), ("timed_ms", C.c_double),
                 ("timed_bytes", C.c_double), ("timed_flops", C.c_double),
-                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64)]
+                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64), ("span_ms", C.c_double)]
 
 
 # exported symbols (tests/test_abi.py checks them against include/bm.h)

@@ -152,6 +152,7 @@ struct Task {
 struct TimedLaunch {
   cudaEvent_t beg, end;
   double bytes, flops;
+  int b;
 };
 
 struct Engine {
@@ -202,6 +203,9 @@ struct Engine {
   int direct_flip = 0;
   std::vector<TimedLaunch> ev_pool;
   int ev_head = 0;
+  unsigned long long* spans = nullptr;  // device: 64 span slots + accumulator (time_kernels)
+  unsigned long long span_base[2] = {0, 0};
+  uint64_t launches_base = 0;
 
   bool device() const { return cfg.clock != BM_CLOCK_DRY; }
   size_t elem() const { return cfg.precision == BM_PREC_BF16 ? 2 : 4; }

@@ -62,6 +62,8 @@ struct StepArgs {
   unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
   unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)
   int pdl;                    // launch with programmatic dependent launch (overlap setup)
+  unsigned long long* span;   // time_kernels: slot {min CTA start, CTAs done} (device memory)
+  unsigned long long* span_acc;  // {sum of launch spans in ns, launches}: last CTA adds
 };
 
 // bf16 / tcgen05 path (cell_step_sm100.cu). a.W: weights in the stage-tile layout

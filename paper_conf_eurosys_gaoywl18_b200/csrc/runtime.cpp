@@ -112,7 +112,10 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
     const int i = e.ev_head;
     e.ev_head = (e.ev_head + 1) % static_cast<int>(e.ev_pool.size());
     tl = &e.ev_pool[i];
+    tl->b = b;
     algo_cost(e, c, b, proj, &tl->bytes, &tl->flops);
+    a.span = e.spans + 2 * (e.stats.kernel_launches % 64);  // 64 slots: PDL overlaps <= 2 launches
+    a.span_acc = e.spans + 128;
     CK(cudaEventRecord(tl->beg, e.stream));
     if (ev_out) *ev_out = i;
   }
@@ -358,6 +361,7 @@ static void free_device(Engine& e) {
     cudaEventDestroy(t.beg);
     cudaEventDestroy(t.end);
   }
+  cudaFree(e.spans);
   if (e.stream) cudaStreamDestroy(e.stream);
 }
 
@@ -423,6 +427,13 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       return fail(BM_E_CUDA);
     if (c.time_kernels) {
       E.ev_pool.resize(4096);
+      // device-side launch spans: 64 slots {start, ctas} + accumulator {ns, launches}
+      if (dalloc(&E.spans, 2 * 64 + 2) != cudaSuccess ||
+          cudaMemsetAsync(E.spans, 0xFF, 2 * 64 * 8, E.stream) != cudaSuccess)
+        return fail(BM_E_NOMEM);
+      for (int i = 0; i < 64; ++i)
+        if (cudaMemsetAsync(E.spans + 2 * i + 1, 0, 8, E.stream) != cudaSuccess) return fail(BM_E_CUDA);
+      if (cudaMemsetAsync(E.spans + 128, 0, 16, E.stream) != cudaSuccess) return fail(BM_E_CUDA);
       for (TimedLaunch& t : E.ev_pool) {
         if (cudaEventCreate(&t.beg) != cudaSuccess || cudaEventCreate(&t.end) != cudaSuccess)
           return fail(BM_E_CUDA);
@@ -913,13 +924,29 @@ bm_status bm_tokens(bm_engine* h, const int32_t* slots, int n, int32_t* inout, i
 
 bm_status bm_get_stats(bm_engine* h, bm_stats* out) {
   if (h == nullptr || out == nullptr) return BM_E_INVAL;
-  *out = reinterpret_cast<Engine*>(h)->stats;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  *out = e.stats;
+  out->kernel_launches = e.stats.kernel_launches - e.launches_base;
+  if (e.spans != nullptr) {  // device-side spans accumulated since the last reset
+    unsigned long long acc[2] = {0, 0};
+    CK(cudaStreamSynchronize(e.stream));
+    CK(cudaMemcpy(acc, e.spans + 128, 16, cudaMemcpyDeviceToHost));
+    out->span_ms = (acc[0] - e.span_base[0]) * 1e-6;
+  }
   return BM_OK;
 }
 
 bm_status bm_reset_stats(bm_engine* h) {
   if (h == nullptr) return BM_E_INVAL;
-  reinterpret_cast<Engine*>(h)->stats = bm_stats{};
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  const uint64_t launches = e.stats.kernel_launches;  // keeps the span slot rotation aligned
+  e.stats = bm_stats{};
+  e.stats.kernel_launches = launches;
+  e.launches_base = launches;
+  if (e.spans != nullptr) {
+    CK(cudaStreamSynchronize(e.stream));
+    CK(cudaMemcpy(e.span_base, e.spans + 128, 16, cudaMemcpyDeviceToHost));
+  }
   return BM_OK;
 }
 
