@@ -291,18 +291,14 @@ def main():
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    from paper_conf_eurosys_gaoywl18_b200 import bm
+    from paper_conf_eurosys_gaoywl18_b200 import bm, shard
 
     wl = a.workload
     n_req = a.reqs or WL[wl]["reqs"]
     # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink), never again
     w = make_weights(wl)
     if dist is not None:
-        for name, arr in weight_arrays(w):
-            t = torch.from_numpy(arr).cuda() if rank == 0 else torch.empty(arr.shape, dtype=torch.float32,
-                                                                            device="cuda")
-            dist.broadcast(t, src=0)
-            arr[...] = t.cpu().numpy()
+        shard.broadcast_arrays(weight_arrays(w), dist, device=torch.device("cuda", local))
     e, cells = build_engine(bm, wl, w, local, max_requests=max(n_req, 1 << 15) + 64, lookahead=a.lookahead)
     stream = torch.cuda.ExternalStream(e.stream(), device=torch.device("cuda", local))
 
@@ -312,14 +308,10 @@ def main():
             dist.barrier()
 
     def allmax(x):
-        if dist is None:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return shard.reduce_max(x, dist, device=torch.device("cuda", local))
 
     # ---- calibrate saturation: every request of a trace arrives at t = 0
-    burst = make_trace(wl, n_req, None, seed=7 + rank)
+    burst = make_trace(wl, n_req, None, seed=shard.rank_seed(7, rank))
     pb = e.prepare_requests(burst, cells)
     run_trace(e, pb, n_req)                      # warm (also JIT of nothing: all AOT)
     dt, _ = run_trace(e, pb, n_req)
@@ -333,7 +325,7 @@ def main():
         for frac in (0.05, 0.1, 0.2, 0.35, 0.5, 0.65, 0.8, 0.9, 1.0, 1.1):
             lam = frac * mu
             n_pt = int(max(2000, min(n_req, lam * 0.25)))
-            tr = make_trace(wl, n_pt, lam, seed=100 + rank)
+            tr = make_trace(wl, n_pt, lam, seed=shard.rank_seed(100, rank))
             p = e.prepare_requests(tr, cells)
             wall, lat = run_trace(e, p, n_pt)
             p50, p90, p99 = (allmax(pct(lat, q)) for q in (50, 90, 99))
@@ -347,7 +339,7 @@ def main():
         if lam_star is None:
             lam_star = 0.05 * mu
     # ---- timed steps at lambda*
-    trace = make_trace(wl, n_req, lam_star, seed=1000 + rank)
+    trace = make_trace(wl, n_req, lam_star, seed=shard.rank_seed(1000, rank))
     prep = e.prepare_requests(trace, cells)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
     for _ in range(a.warmup):
@@ -372,11 +364,11 @@ def main():
             lats.append(np.array([c.t_done - c.t_arrival for c in comp]))
     barrier()
     st = e.stats()
-    lat = np.concatenate(lats)
+    lat = shard.gather_samples(np.concatenate(lats), dist, device=torch.device("cuda", local))
     t_max = allmax(dev_ms / 1e3)
     total = n_req * a.steps * world
     value = total / t_max
-    p50, p90, p99 = (allmax(pct(lat, q)) for q in (50, 90, 99))
+    p50, p90, p99 = shard.percentiles(lat)   # over the union of all ranks' requests
     # ---- e2e: public API with host buffers (submit from host, descriptors H2D every Schedule
     #      call inside bm_run, final h rows D2H), timed on the host clock around the whole thing
     e2, cells2 = build_engine(bm, wl, w, local, max_requests=n_req + 64, lookahead=a.lookahead,

@@ -296,7 +296,6 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
-  if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
   if (tid == 0) {
     for (int s = 0; s < kMaxStages; ++s) {
       mbar_init(full0 + 8 * s, kProducerThreads + 1);  // gather threads + the TMA thread
@@ -322,6 +321,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (warp < 8) {
     // ================================================================ activation gather (A6)
     pdl_wait();  // rows, pool h/c and feed tokens are written by earlier launches / copies
+    // device span starts when the launch's dependent work may begin (after the PDL wait)
+    if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
     for (int c = tid; c < kMaxCols; c += kProducerThreads) {
       const __nv_bfloat16* s0 = nullptr;
       const __nv_bfloat16* s1 = nullptr;
