@@ -85,6 +85,7 @@ int main(int argc, char** argv) {
   const int stages = argc > 4 ? atoi(argv[4]) : 4;
   const int l2_resident = argc > 5 ? atoi(argv[5]) : 1;  // 1: same bytes every launch
   const int mode = argc > 6 ? atoi(argv[6]) : 0;          // 0 bulk, 1 cp.async, 2 ldg
+  const int share = argc > 7 ? atoi(argv[7]) : 1 << 30;   // CTAs i and i+share.. read the same bytes
   const size_t total = per_cta * ctas;
   const size_t buf_bytes = l2_resident ? total : (size_t)2 << 30;
   uint8_t* src;
@@ -104,7 +105,7 @@ int main(int argc, char** argv) {
     cudaEventRecord(a);
     for (int it = 0; it < iters; ++it) {
       const uint8_t* s = l2_resident ? src : src + ((size_t)it * total) % (buf_bytes - total);
-      if (mode == 0) ingest<<<ctas, 32, smem>>>(s, per_cta, chunk, stages, 1 << 30, sink);
+      if (mode == 0) ingest<<<ctas, 32, smem>>>(s, per_cta, chunk, stages, share, sink);
       else ingest_threads<<<ctas, 256, smem>>>(s, per_cta, chunk, stages, mode, sink);
     }
     cudaEventRecord(b);
@@ -114,7 +115,7 @@ int main(int argc, char** argv) {
     if (ms < best) best = ms;
   }
   const double us = best * 1e3 / iters;
-  printf("{\"mode\": %d, \"ctas\": %d, \"per_cta\": %zu, \"chunk\": %d, \"stages\": %d, \"l2\": %d, \"us\": %.2f, \"GBps\": %.1f, \"err\": \"%s\"}\n",
-         mode, ctas, per_cta, chunk, stages, l2_resident, us, total / us / 1e3, cudaGetErrorString(cudaGetLastError()));
+  printf("{\"share\": %d, \"mode\": %d, \"ctas\": %d, \"per_cta\": %zu, \"chunk\": %d, \"stages\": %d, \"l2\": %d, \"us\": %.2f, \"GBps\": %.1f, \"err\": \"%s\"}\n",
+         share, mode, ctas, per_cta, chunk, stages, l2_resident, us, total / us / 1e3, cudaGetErrorString(cudaGetLastError()));
   return 0;
 }
