@@ -57,10 +57,13 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="lstm", choices=["lstm", "seq2seq", "tree"])
     p.add_argument("--reqs", type=int, default=0, help="requests per step (0 = per-workload default)")
-    p.add_argument("--p90-ms", type=float, default=12.0)
+    p.add_argument("--p90-ms", type=float, default=0.0,
+                   help="p90 bound; 0 = per-workload default (12 ms, L489; Seq2Seq: the knee, "
+                        "2x the lowest-load p90, since Fig. 13's values are not legible)")
     p.add_argument("--rate", type=float, default=0.0, help="skip the sweep, use this offered rate")
-    p.add_argument("--lookahead", type=int, default=8,
-                   help="schedule when <= k tasks are outstanding (0 = the paper's idle-only)")
+    p.add_argument("--lookahead", type=int, default=-1,
+                   help="schedule when <= k tasks are outstanding (0 = the paper's idle-only); "
+                        "-1 = per-workload default")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--out", default="")
@@ -70,12 +73,14 @@ def parse():
 # ------------------------------------------------------------------------------ workloads
 WL = {
     "lstm": dict(config="BASELINE configs[1]: 1-layer LSTM h=1024, WMT-like lengths, Poisson arrivals, "
-                        "bmax 512, 1 B200", hidden=1024, layers=1, vocab=32768, reqs=20000),
+                        "bmax 512, 1 B200", hidden=1024, layers=1, vocab=32768, reqs=20000,
+                 p90_ms=12.0, lookahead=2),
     "seq2seq": dict(config="BASELINE configs[2]: Seq2Seq 4+4 layer LSTM h=1024, vocab 32768, greedy "
                            "decode, encoder/decoder bmax 512/256", hidden=1024, layers=4, vocab=32768,
-                    reqs=4000),
+                    reqs=4000, p90_ms=None, lookahead=1),
     "tree": dict(config="BASELINE configs[3]: TreeLSTM h=1024, TreeBank-shaped binary trees, leaf/internal "
-                        "cells batched separately, bmax 64", hidden=1024, layers=1, vocab=32768, reqs=6000),
+                        "cells batched separately, bmax 64", hidden=1024, layers=1, vocab=32768, reqs=6000,
+                 p90_ms=12.0, lookahead=2),
 }
 
 
@@ -295,6 +300,8 @@ def main():
 
     wl = a.workload
     n_req = a.reqs or WL[wl]["reqs"]
+    if a.lookahead < 0:
+        a.lookahead = WL[wl]["lookahead"]
     # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink), never again
     w = make_weights(wl)
     if dist is not None:
@@ -318,10 +325,11 @@ def main():
     mu = n_req / dt
     # ---- load sweep (open loop), untimed: highest rate whose p90 <= bound
     curve = []
+    bound_kind = "absolute"
     if a.rate > 0:
         lam_star = a.rate
+        bound_ms = a.p90_ms or WL[wl]["p90_ms"] or 12.0
     else:
-        lam_star = None
         for frac in (0.05, 0.1, 0.2, 0.35, 0.5, 0.65, 0.8, 0.9, 1.0, 1.1):
             lam = frac * mu
             n_pt = int(max(2000, min(n_req, lam * 0.25)))
@@ -329,15 +337,19 @@ def main():
             p = e.prepare_requests(tr, cells)
             wall, lat = run_trace(e, p, n_pt)
             p50, p90, p99 = (allmax(pct(lat, q)) for q in (50, 90, 99))
-            thr = allmax(n_pt / wall)
             curve.append({"offered": lam, "achieved": n_pt / wall, "p50_ms": p50 * 1e3, "p90_ms": p90 * 1e3,
                           "p99_ms": p99 * 1e3})
-            if p90 * 1e3 <= a.p90_ms:
-                lam_star = lam
-            elif lam_star is not None:
-                break
-        if lam_star is None:
-            lam_star = 0.05 * mu
+        bound_ms = a.p90_ms or WL[wl]["p90_ms"]
+        if not bound_ms:   # the knee: 2x the lowest-load p90
+            bound_ms = 2.0 * curve[0]["p90_ms"]
+            bound_kind = "knee (2x lowest-load p90)"
+
+        def best_under(b):
+            ok = [c["offered"] for c in curve if c["p90_ms"] <= b]
+            return max(ok) if ok else None
+        lam_star = best_under(bound_ms) or curve[0]["offered"]
+        knee_ms = 2.0 * curve[0]["p90_ms"]
+        bounds = {"12ms": best_under(12.0), "knee": best_under(knee_ms), "knee_ms": knee_ms}
     # ---- timed steps at lambda*
     trace = make_trace(wl, n_req, lam_star, seed=shard.rank_seed(1000, rank))
     prep = e.prepare_requests(trace, cells)
@@ -418,7 +430,9 @@ def main():
                 "warmup": a.warmup, "ms_per_step": t_max * 1e3 / a.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
                 "config": {"workload": WL[wl]["config"], "requests_per_step": n_req,
-                           "offered_rate_per_gpu": lam_star, "p90_bound_ms": a.p90_ms,
+                           "offered_rate_per_gpu": lam_star, "p90_bound_ms": bound_ms,
+                           "p90_bound_kind": bound_kind,
+                           "max_offered_rate_under": bounds if a.rate <= 0 else None,
                            "saturation_burst_rate_per_gpu": mu, "lookahead_k": a.lookahead,
                            "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
                                  "step (serving)", "parallelism": f"request-sharded x{world}"},

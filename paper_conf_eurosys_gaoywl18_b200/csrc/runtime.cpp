@@ -72,8 +72,12 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
   a.K0 = c.K0;
   a.K1 = proj ? 0 : c.K1;
   a.U = c.U;
-  a.S = proj ? 1 : c.S;
-  a.kslice = proj ? e.cfg.hidden : c.kslice;
+  // split-K factor per launch (bf16 path): 512-wide K slices up to 256 rows (one wave of
+  // 128-160 CTAs); above that two column blocks with 1024-wide slices keep one wave instead of
+  // two (the wider K slice costs less than a second wave and halves the DSMEM exchange).
+  a.S = c.S;
+  if (e.cfg.precision == BM_PREC_BF16 && b > 256 && c.S >= 4) a.S = c.S / 2;
+  a.kslice = (c.K0 + c.K1) / a.S;
   if (proj) {
     a.S = 1;
     a.kslice = e.cfg.hidden;

@@ -26,7 +26,7 @@ def main():
     prec = bm.PREC_FP32 if a.fp32 else bm.PREC_BF16
     bf = not a.fp32
     e = bm.Engine(precision=prec, hidden=H, pool_layers=1, max_slots=8192, max_requests=8192,
-                  max_decode_len=4)
+                  max_decode_len=4, time_kernels=1)
     if a.cell in ("lstm", "proj"):
         w = gen.lstm_stack_weights(H, 1, V, 0, projection=a.cell == "proj", bf16=bf)
         kind = bm.CELL_LSTM_PROJ if a.cell == "proj" else bm.CELL_LSTM
@@ -54,6 +54,7 @@ def main():
         for _ in range(5):
             e.cell_step(cid, rows, sync=False)
         torch.cuda.synchronize()
+        e.reset_stats()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         for _ in range(a.iters):
@@ -61,6 +62,9 @@ def main():
         ev1.record(stream)
         ev1.synchronize()
         us = ev0.elapsed_time(ev1) * 1e3 / a.iters
+        st = e.stats()
+        launches = max(1, st["timed_launches"])
+        span_us = st["span_ms"] * 1e3 / launches       # device: first CTA start .. last CTA end
         if a.cell == "proj":
             # LSTM layer + projection per call; report the sum
             byts = (rows_w * K * el + b * 14336) + (V * H * el + b * (2 * H + 8))
@@ -69,7 +73,9 @@ def main():
             per_row = K * el + H * el + H * 4 + (H * 4 if a.cell == "lstm" else 2 * H * 4 if a.cell == "internal" else 0)
             byts = rows_w * K * el + rows_w * 4 + b * per_row
             flops = 2 * b * K * rows_w
-        r = {"cell": a.cell, "b": b, "us": us, "GBps": byts / us / 1e3, "TFLOPs": flops / us / 1e6}
+        r = {"cell": a.cell, "b": b, "us_per_call": us, "span_us": span_us,
+             "GBps_span": byts / span_us / 1e3 if span_us > 0 else None,
+             "TFLOPs_span": flops / span_us / 1e6 if span_us > 0 else None}
         print(json.dumps(r), flush=True)
         out.append(r)
     if a.out:
