@@ -72,6 +72,12 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   while (!mbar_try_wait(bar, parity)) {
   }
 }
+// Warp-wide wait with ONE polling lane: 256 threads polling the same mbarrier measurably slow
+// down the barrier traffic of the MMA issuer (0.3 us per main-loop step instead of ~0.05 us).
+__device__ __forceinline__ void mbar_wait_warp(uint32_t bar, uint32_t parity) {
+  if ((threadIdx.x & 31) == 0) mbar_wait(bar, parity);
+  __syncwarp();
+}
 // Contiguous global -> shared bulk copy (TMA engine), completion counted on an mbarrier.
 __device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
   asm volatile(
@@ -196,19 +202,29 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
-// Shared-memory plan (identical on host and device). Small tasks (npad <= 128) keep the
-// footprint near 100 KB so two CTAs fit per SM (the next launch's CTAs can start under PDL while
-// this one drains); larger tasks take ~200 KB. Stage depth matters little (the per-SM ingest
-// rate, not latency, bounds the stream: tools/ingest_bench.cu), so the budget decides it.
-__host__ __device__ __forceinline__ int stage_bytes(int npad) { return kWStageBytes + npad * 128; }
-__host__ __device__ __forceinline__ int stages_for(int npad) {
-  const int budget = npad <= 128 ? 96 * 1024 : 192 * 1024;
-  const int n = budget / stage_bytes(npad);
-  return n < kMaxStages ? (n < 2 ? 2 : n) : kMaxStages;
+// Shared-memory plan (identical on host and device).
+// The weight stream and the activation gather use separate rings:
+//  * weights: contiguous pre-swizzled tiles, moved by the TMA engine in chunks of kWChunkKB
+//    K-blocks (64 KB for 128-row tiles). The per-SM TMA engine completes bulk copies one at a
+//    time, so its throughput grows with the chunk size (8 KB: 23 GB/s/SM, 16 KB: 42, 32 KB: 64,
+//    64 KB: 85, tools/ingest_bench.cu) and not with the number in flight; a 2-chunk ring covers
+//    the whole 512-wide K slice of a split-K CTA.
+//  * activations: one 64-wide K block per stage, gathered by 256 threads with cp.async (the
+//    LSU path runs beside the TMA engine).
+constexpr int kWChunkMax = 4;           // K blocks per weight chunk, large tasks (64 KB chunks)
+constexpr int kWRing = 2;               // weight chunks in the ring
+// Small tasks (npad <= 128) use 32 KB weight chunks and a 32 KB activation ring so the CTA fits
+// in ~100 KB and two CTAs share an SM: under PDL the next launch's weight stream and gather
+// overlap this launch's split-K epilogue. Larger tasks use 64 KB chunks and a 64 KB ring.
+__host__ __device__ __forceinline__ int w_chunk_blocks(int npad) { return npad <= 128 ? 2 : kWChunkMax; }
+__host__ __device__ __forceinline__ int x_ring_bytes(int npad) { return npad <= 128 ? 32 * 1024 : 64 * 1024; }
+__host__ __device__ __forceinline__ int x_stages_for(int npad) {
+  const int n = x_ring_bytes(npad) / (npad * 128);
+  return n < 2 ? 2 : (n > kMaxStages ? kMaxStages : n);
 }
-// stage ring, reused after the main loop for the partial / logits tile (<= 129 x npad fp32)
+// weight ring + activation ring, reused after the main loop for the partial / logits tile
 __host__ __device__ __forceinline__ int region_bytes(int npad) {
-  const int a = stages_for(npad) * stage_bytes(npad);
+  const int a = kWRing * w_chunk_blocks(npad) * kWStageBytes + x_stages_for(npad) * npad * 128;
   const int b = 129 * npad * 4 + 4 * 128 * 4;
   return a > b ? a : b;
 }
@@ -227,7 +243,7 @@ __device__ __forceinline__ void phase_mark(const StepArgs& p, int i) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-    p.phase[cta * 8 + i] = t;
+    p.phase[cta * 16 + i] = t;
   }
 }
 
@@ -262,7 +278,7 @@ __device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const
 
 // ------------------------------------------------------------------ the kernel
 template <int EPI>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kThreads, 2)
     cell_step_sm100_kernel(const __grid_constant__ StepArgs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -279,27 +295,38 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int npad = (ncols + 15) & ~15;
   const int nk = p.kslice / kBK;
   const int k_begin = static_cast<int>(rank) * p.kslice;
-  const int kStages = p.max_stages > 0 ? min(p.max_stages, stages_for(npad)) : stages_for(npad);
+  const int kStages = p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad)) : x_stages_for(npad);
+  const int wcb = w_chunk_blocks(npad);                   // ring slot capacity in K blocks
+  const int kpc = min(wcb, nk);                           // K blocks per weight chunk
+  const int n_chunks = (nk + kpc - 1) / kpc;
+  const int wblk_bytes = tile_rows * 128;                 // one K block of this CTA's weight tile
 
-  // shared memory: [tail: row sources + barriers][stage ring: W tiles | X tiles]
+  // shared memory: [tail: row sources + barriers][weight ring | activation ring]
   const __nv_bfloat16** src_tab = reinterpret_cast<const __nv_bfloat16**>(base);  // [2][256]
   uint64_t* bars = reinterpret_cast<uint64_t*>(base + 2 * kMaxCols * sizeof(void*));
-  const uint32_t full0 = smem_u32(bars);
-  const uint32_t empty0 = smem_u32(bars + kMaxStages);
-  const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 1);
+  const uint32_t full0 = smem_u32(bars);                            // activation stage full
+  const uint32_t empty0 = smem_u32(bars + kMaxStages);              // activation stage free
+  const uint32_t wfull0 = smem_u32(bars + 2 * kMaxStages);          // weight chunk landed
+  const uint32_t wempty0 = smem_u32(bars + 2 * kMaxStages + kWRing);  // weight chunk free
+  const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages + 2 * kWRing);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 2 * kWRing + 1);
   int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
   uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
-  uint8_t* w_st = smem;                                   // kStages x 16 KB
-  uint8_t* x_st = smem + kStages * kWStageBytes;          // kStages x npad x 128 B
+  uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
+  uint8_t* x_st = smem + kWRing * wcb * kWStageBytes;     // kStages x npad x 128 B
   const int x_stage_bytes = npad * 128;
 
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
+  if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 16 + 14] = clock64();
   if (tid == 0) {
     for (int s = 0; s < kMaxStages; ++s) {
-      mbar_init(full0 + 8 * s, kProducerThreads + 1);  // gather threads + the TMA thread
+      mbar_init(full0 + 8 * s, 1);  // one gather thread arrives after a producer-wide barrier
       mbar_init(empty0 + 8 * s, 1);
+    }
+    for (int s = 0; s < kWRing; ++s) {
+      mbar_init(wfull0 + 8 * s, 1);   // the TMA thread's arrive.expect_tx
+      mbar_init(wempty0 + 8 * s, 1);
     }
     mbar_init(done_bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -323,6 +350,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     pdl_wait();  // rows, pool h/c and feed tokens are written by earlier launches / copies
     // device span starts when the launch's dependent work may begin (after the PDL wait)
     if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
+    if (tid == 0) phase_mark(p, 8);
     for (int c = tid; c < kMaxCols; c += kProducerThreads) {
       const __nv_bfloat16* s0 = nullptr;
       const __nv_bfloat16* s1 = nullptr;
@@ -335,6 +363,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       src_tab[kMaxCols + c] = s1;
     }
     named_bar(1, kProducerThreads);
+    if (tid == 0) phase_mark(p, 9);
     // Every stage's cp.async group stays in flight until the ring is full; a stage is handed
     // to the MMA (full barrier) once its group has landed and been made visible to the
     // async proxy. lag = stages - 1 keeps the whole ring in flight without deadlock.
@@ -343,16 +372,20 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int kb = 0; kb < nk; ++kb) {
       const int s = kb % kStages;
       const int round = kb / kStages;
-      if (round > 0) mbar_wait(empty0 + 8 * s, (round - 1) & 1);
+      if (round > 0) mbar_wait_warp(empty0 + 8 * s, (round - 1) & 1);
       const int k = k_begin + kb * kBK;
       const int seg = k >= p.K0 ? 1 : 0;
       const int kk = k - seg * p.K0;
       const uint32_t xs = smem_u32(x_st + s * x_stage_bytes);
       const __nv_bfloat16** tab = src_tab + seg * kMaxCols;
+      if (p.experiment & 4) {  // diagnostics: no gather at all, hand the stage over at once
+        if (tid == 0) mbar_arrive(full0 + 8 * s);
+        continue;
+      }
       for (int q = tid; q < npad * 8; q += kProducerThreads) {
         const int row = q >> 3;
         const int ch = q & 7;
-        const __nv_bfloat16* src = tab[row];
+        const __nv_bfloat16* src = (p.experiment & 1) ? nullptr : tab[row];
         const uint32_t dst = xs + row * 128 + ((ch ^ (row & 7)) << 4);
         if (src != nullptr) {
           cp_async_16(dst, src + kk + ch * 8, 16);
@@ -361,32 +394,47 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
       cp_async_commit();
+      if (tid == 0 && kb == 0) phase_mark(p, 10);
       if (kb >= lag) {
+        // every producer's copies of stage kb - lag have landed and are visible to the async
+        // proxy; one thread then hands the stage to the MMA (256 release-arrives per stage
+        // measured ~0.3 us per hand-off, a named barrier + one arrive ~0.05 us)
         cp_async_wait_dyn(lag);
         fence_proxy_async();
-        mbar_arrive(full0 + 8 * ((kb - lag) % kStages));
+        named_bar(1, kProducerThreads);
+        if (tid == 0 && kb == lag) phase_mark(p, 11);
+        if (tid == 0) mbar_arrive(full0 + 8 * ((kb - lag) % kStages));
       }
     }
     cp_async_wait<0>();
     fence_proxy_async();
-    for (int kb = max(0, nk - lag); kb < nk; ++kb) mbar_arrive(full0 + 8 * (kb % kStages));
+    named_bar(1, kProducerThreads);
+    if (!(p.experiment & 4) && tid == 0)
+      for (int kb = max(0, nk - lag); kb < nk; ++kb) mbar_arrive(full0 + 8 * (kb % kStages));
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
     // Weights are read-only: streaming starts before griddepcontrol.wait (PDL overlap).
     if (lane == 0) {
-      const int wbytes = tile_rows * 128;
       const int kblocks = (p.K0 + p.K1) / kBK;
       const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
-                            (static_cast<size_t>(blockIdx.y) * kblocks + k_begin / kBK) * wbytes;
-      for (int kb = 0; kb < nk; ++kb) {
-        const int s = kb % kStages;
-        const int round = kb / kStages;
-        if (round > 0) mbar_wait(empty0 + 8 * s, (round - 1) & 1);
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(full0 + 8 * s),
-                     "r"(wbytes)
+                            (static_cast<size_t>(blockIdx.y) * kblocks + k_begin / kBK) * wblk_bytes;
+      for (int c = 0; c < n_chunks; ++c) {
+        const int s = c % kWRing;
+        const int round = c / kWRing;
+        if (round > 0) mbar_wait(wempty0 + 8 * s, (round - 1) & 1);
+        const int nblk = min(kpc, nk - c * kpc);
+        const uint32_t bytes = static_cast<uint32_t>(nblk * wblk_bytes);
+        if (p.experiment & 2) {  // diagnostics: no weight traffic
+          mbar_arrive(wfull0 + 8 * s);
+          continue;
+        }
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(wfull0 + 8 * s),
+                     "r"(bytes)
                      : "memory");
-        bulk_load(smem_u32(w_st + s * kWStageBytes), wsrc + static_cast<size_t>(kb) * wbytes, wbytes,
-                  full0 + 8 * s);
+        // one chunk = nblk consecutive K blocks (contiguous in the stage-tile layout); block i
+        // lands at i * wblk_bytes (a multiple of 1024: the 128B-swizzle atom stays aligned)
+        bulk_load(smem_u32(w_ring + s * wcb * kWStageBytes),
+                  wsrc + static_cast<size_t>(c) * kpc * wblk_bytes, bytes, wfull0 + 8 * s);
       }
     }
     __syncwarp();
@@ -395,25 +443,34 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint32_t idesc = idesc_bf16(128, npad);
     for (int kb = 0; kb < nk; ++kb) {
       const int s = kb % kStages;
-      mbar_wait(full0 + 8 * s, (kb / kStages) & 1);
+      const int c = kb / kpc;
+      const int ws = c % kWRing;
+      if (kb % kpc == 0) mbar_wait_warp(wfull0 + 8 * ws, (c / kWRing) & 1);
+      if (lane == 0 && kb == 0) phase_mark(p, 13);
+      mbar_wait_warp(full0 + 8 * s, (kb / kStages) & 1);
       tc_fence_after();
       if (lane == 0 && kb == 0) phase_mark(p, 6);
       if (lane == 0 && kb == nk - 1) phase_mark(p, 7);
+      if (lane == 0 && kb == 1) phase_mark(p, 12);
       if (lane == 0) {
-        const uint64_t a = sdesc_sw128(smem_u32(w_st + s * kWStageBytes));
+        const uint64_t a =
+            sdesc_sw128(smem_u32(w_ring + ws * wcb * kWStageBytes + (kb % kpc) * wblk_bytes));
         const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes));
+        if (!(p.experiment & 8)) {  // diagnostics bit 8: no MMA instructions
 #pragma unroll
-        for (int k = 0; k < kBK / 16; ++k) {
-          mma_bf16(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
+          for (int k = 0; k < kBK / 16; ++k) {
+            mma_bf16(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
+          }
         }
         mma_commit(empty0 + 8 * s);
+        if (kb % kpc == kpc - 1 || kb == nk - 1) mma_commit(wempty0 + 8 * ws);
         if (kb == nk - 1) mma_commit(done_bar);
       }
       __syncwarp();
     }
   }
   if (warp < 8) {
-    mbar_wait(done_bar, 0);
+    mbar_wait_warp(done_bar, 0);
     tc_fence_after();
     if (tid == 0) phase_mark(p, 2);
   }
@@ -586,6 +643,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (tid == 0) phase_mark(p, 4);
     cluster_sync();  // B: peers may read this CTA's partials until here
     if (tid == 0) phase_mark(p, 5);
+    if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 16 + 15] = clock64();
     if (p.signal != nullptr) {  // completion signal (A12) fused into the task's last CTA
       __threadfence();
       __syncthreads();
@@ -624,7 +682,9 @@ template <int EPI>
 cudaError_t launch_impl(const StepArgs& a, cudaStream_t st) {
   static bool configured = false;
   if (!configured) {
-    const int max_smem = 1024 + kTailBytes + region_bytes(kMaxCols);
+    const int max_smem = 1024 + kTailBytes + region_bytes(16) > 1024 + kTailBytes + region_bytes(kMaxCols)
+                             ? 1024 + kTailBytes + region_bytes(16)
+                             : 1024 + kTailBytes + region_bytes(kMaxCols);
     cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
     if (e != cudaSuccess) return e;

@@ -58,6 +58,8 @@ struct StepArgs {
   float* logits;              // debug [max_requests][max_decode][V] or null
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer at phase boundaries, or null
   int max_stages;             // experiments (BM_MAX_STAGES): cap on pipeline stages, 0 = default
+  int experiment;             // diagnostics (BM_EXPERIMENT) bit 1: no activation reads (zero
+                              // fill), bit 2: no weight copies; results are garbage
   // launch path
   unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
   unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)

@@ -108,11 +108,18 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
   a.phase = e.phase_dev;
   static const int max_stages = getenv("BM_MAX_STAGES") ? atoi(getenv("BM_MAX_STAGES")) : 0;
   a.max_stages = max_stages;
+  static const int experiment = getenv("BM_EXPERIMENT") ? atoi(getenv("BM_EXPERIMENT")) : 0;
+  a.experiment = experiment;
   a.signal = signal;
   a.sig_ctas = e.sig_ctas;
-  a.pdl = 1;
+  static const int no_pdl = getenv("BM_NO_PDL") ? atoi(getenv("BM_NO_PDL")) : 0;
+  a.pdl = no_pdl ? 0 : 1;
   TimedLaunch* tl = nullptr;
-  if (e.cfg.time_kernels && !e.ev_pool.empty()) {
+  // events serialise the stream and so disable PDL overlap around the launches they bracket:
+  // time a sample (every kTimeEvery-th launch) instead of every launch
+  static const int time_every = getenv("BM_TIME_EVERY") ? atoi(getenv("BM_TIME_EVERY")) : 8;
+  const bool sample = (e.stats.kernel_launches % (time_every > 0 ? time_every : 1)) == 0;
+  if (e.cfg.time_kernels && !e.ev_pool.empty() && sample) {
     const int i = e.ev_head;
     e.ev_head = (e.ev_head + 1) % static_cast<int>(e.ev_pool.size());
     tl = &e.ev_pool[i];
@@ -824,23 +831,30 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
   CK(cudaMemcpyAsync(e.direct_rows + e.direct_flip * 4096, stage, sizeof(RowDesc) * b, cudaMemcpyHostToDevice, e.stream));
   CK(cudaEventRecord(e.direct_ev[e.direct_flip], e.stream));
   RowDesc* rows_dev = e.direct_rows + e.direct_flip * 4096;
+  // diagnostics: BM_REPEAT=n launches the step n times back to back (steady-state throughput
+  // with PDL overlap between consecutive launches; the state advances n steps)
+  static const int repeat = getenv("BM_REPEAT") ? atoi(getenv("BM_REPEAT")) : 1;
+  for (int rep = 1; rep < repeat; ++rep) {
+    bm_status s0 = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
+    if (s0 != BM_OK) return s0;
+  }
   // diagnostics: BM_PHASE_DUMP=<file> records per-CTA phase timestamps of every direct step
   static const char* dump = getenv("BM_PHASE_DUMP");
-  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 8 * 4096));
-  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 8 * 4096, e.stream));
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 16 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 16 * 4096, e.stream));
   bm_status s = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
   if (s != BM_OK) return s;
   if (!async || e.phase_dev) CK(cudaStreamSynchronize(e.stream));
   if (e.phase_dev) {
-    std::vector<unsigned long long> h(8 * 4096);
+    std::vector<unsigned long long> h(16 * 4096);
     CK(cudaMemcpy(h.data(), e.phase_dev, h.size() * 8, cudaMemcpyDeviceToHost));
     FILE* f = fopen(dump, "a");
     if (f) {
       fprintf(f, "step b=%d cell=%d\n", b, cell_id);
       for (int i = 0; i < 4096; ++i)
-        if (h[i * 8]) {
+        if (h[i * 16]) {
           fprintf(f, "%d", i);
-          for (int k = 0; k < 8; ++k) fprintf(f, " %llu", h[i * 8 + k]);
+          for (int k = 0; k < 16; ++k) fprintf(f, " %llu", h[i * 16 + k]);
           fprintf(f, "\n");
         }
       fclose(f);

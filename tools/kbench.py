@@ -57,13 +57,17 @@ def main():
         e.reset_stats()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
+        import time as _t
+        th0 = _t.perf_counter()
         for _ in range(a.iters):
             e.cell_step(cid, rows, sync=False)
+        th1 = _t.perf_counter()
         ev1.record(stream)
         ev1.synchronize()
         us = ev0.elapsed_time(ev1) * 1e3 / a.iters
         st = e.stats()
-        launches = max(1, st["timed_launches"])
+        reps = int(os.environ.get("BM_REPEAT", "1"))
+        launches = a.iters * reps * (2 if a.cell == "proj" else 1)
         span_us = st["span_ms"] * 1e3 / launches       # device: first CTA start .. last CTA end
         if a.cell == "proj":
             # LSTM layer + projection per call; report the sum
@@ -73,7 +77,8 @@ def main():
             per_row = K * el + H * el + H * 4 + (H * 4 if a.cell == "lstm" else 2 * H * 4 if a.cell == "internal" else 0)
             byts = rows_w * K * el + rows_w * 4 + b * per_row
             flops = 2 * b * K * rows_w
-        r = {"cell": a.cell, "b": b, "us_per_call": us, "span_us": span_us,
+        r = {"cell": a.cell, "b": b, "us_per_call": us, "us_per_step": us / reps, "span_us": span_us,
+             "host_us_per_call": (th1 - th0) * 1e6 / a.iters,
              "GBps_span": byts / span_us / 1e3 if span_us > 0 else None,
              "TFLOPs_span": flops / span_us / 1e6 if span_us > 0 else None}
         print(json.dumps(r), flush=True)

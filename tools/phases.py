@@ -13,7 +13,7 @@ for line in open(sys.argv[1]):
         steps.append(cur)
     else:
         v = [int(x) for x in line.split()]
-        cur["rows"].append(v[1:9])
+        cur["rows"].append(v[1:17])
 for st in steps[-3:]:
     a = np.array(st["rows"], dtype=np.float64)
     t0 = a[:, 0].min()
@@ -23,6 +23,14 @@ for st in steps[-3:]:
     for k in range(1, 6):
         d = (a[:, k] - a[:, k - 1]) / 1e3
         print("  %-8s us: min %.2f med %.2f max %.2f" % (names[k], d.min(), np.median(d), d.max()))
-    for k, nm in ((6, "first stage at MMA (from setup)"), (7, "last stage at MMA (from setup)")):
+    for k, nm in ((8, "producer after PDL wait"), (9, "producer row table done"),
+                  (10, "producer stage 0 issued"), (11, "producer first hand-off"),
+                  (12, "second stage at MMA"), (13, "MMA got weight chunk 0"),
+                  (6, "first stage at MMA (from setup)"), (7, "last stage at MMA (from setup)")):
         d = (a[:, k] - a[:, 1]) / 1e3
         print("  %-32s us: min %.2f med %.2f max %.2f" % (nm, d.min(), np.median(d), d.max()))
+    cyc = a[:, 15] - a[:, 14]
+    ns = a[:, 5] - a[:, 0]
+    ok = (cyc > 0) & (ns > 0)
+    if ok.any():
+        print("  SM clock (clock64 / globaltimer over each CTA): median %.0f MHz" % np.median(cyc[ok] / ns[ok] * 1e3))
