@@ -78,11 +78,16 @@ typedef struct {
   int record_logits;         /* debug: keep every decode step's logits (parity tests)     */
   int time_kernels;          /* 1: CUDA-event time every cell-step launch (bench roofline)*/
   int record_log;            /* 1: keep the task log for bm_read_log (default 1)          */
+  int persistent;            /* 1: bm_run serves an engine whose only cell is a 1-layer   */
+                             /* LSTM with one persistent, weight-stationary kernel (its   */
+                             /* weight slice stays in shared memory; tasks arrive through */
+                             /* a device ring; a grid barrier separates tasks). Ignored   */
+                             /* (regular launches) when the engine is not eligible.       */
 } bm_config;
 
 /* Fill *cfg with defaults: device 0, BF16, WALL, hidden 1024, 1 layer, 65536 slots,
  * 65536 requests, MaxTasksToSubmit 5, Min 1, k 0, max_decode_len 512, keep_results 0,
- * record_log 1. */
+ * record_log 1, persistent 0. */
 void bm_config_default(bm_config* cfg);
 
 /* ---------------------------------------------------------------- cells (bm_load_cell) */

@@ -34,7 +34,8 @@ class Config(C.Structure):
     _fields_ = [(n, C.c_int) for n in (
         "device", "precision", "clock", "hidden", "pool_layers", "max_slots", "max_requests",
         "max_tasks_to_submit", "min_followon_batch", "schedule_when_outstanding_leq",
-        "max_decode_len", "keep_results", "record_logits", "time_kernels", "record_log")]
+        "max_decode_len", "keep_results", "record_logits", "time_kernels", "record_log",
+        "persistent")]
 
 
 class CellDesc(C.Structure):

@@ -19,7 +19,8 @@ CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "libbm.so")
 BUILD = os.path.join(HERE, "_build")
 
-SOURCES = ["cell_step_sm100.cu", "cell_step_simt.cu", "scheduler.cpp", "runtime.cpp"]
+SOURCES = ["cell_step_sm100.cu", "lstm_persistent_sm100.cu", "cell_step_simt.cu", "scheduler.cpp",
+           "runtime.cpp"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
@@ -38,7 +39,7 @@ def _stale(target: str, deps) -> bool:
 
 
 def _headers():
-    hs = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".h")]
+    hs = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".h", ".cuh"))]
     return hs + [os.path.join(ROOT, "include", "bm.h")]
 
 

@@ -201,6 +201,15 @@ struct Engine {
   RowDesc* direct_host = nullptr;  // pinned staging of bm_cell_step rows (double buffered)
   cudaEvent_t direct_ev[2] = {nullptr, nullptr};
   int direct_flip = 0;
+  // persistent weight-stationary LSTM (bm_config.persistent)
+  bool persistent_active = false;
+  cudaStream_t copy_stream = nullptr;  // ring copies while the persistent kernel owns `stream`
+  TaskHdr* hdr_dev = nullptr;
+  TaskHdr* hdr_host = nullptr;         // pinned staging
+  int hdr_ring = 256;
+  unsigned int* gbar = nullptr;
+  int* perr = nullptr;
+  uint64_t run_base = 0;               // launch index of the run's first task
   std::vector<TimedLaunch> ev_pool;
   int ev_head = 0;
   unsigned long long* spans = nullptr;  // device: 64 span slots + accumulator (time_kernels)

@@ -68,6 +68,35 @@ struct StepArgs {
   unsigned long long* span_acc;  // {sum of launch spans in ns, launches}: last CTA adds
 };
 
+// Persistent weight-stationary LSTM engine (lstm_persistent_sm100.cu).
+struct TaskHdr {
+  int32_t seq;      // run-local task index; the kernel polls for the value it expects
+  int32_t b;        // rows; -1 = stop
+  int32_t row_off;  // first row in the device descriptor ring
+  int32_t flags;
+};
+struct PersistArgs {
+  int H, K, K0, S, kslice, n_slots, res_layers, hdr_ring;
+  const TaskHdr* hdr;
+  const RowDesc* rows;
+  const void* E;
+  void* h_pool;
+  float* c_pool;
+  int* tok;
+  const void* W;              // stage-tile layout (launch_pack_tiles)
+  const float* bias;
+  float* res_h;
+  float* res_c;
+  unsigned int* gbar;         // grid-barrier counter (zero at launch)
+  int* err;                   // set to 1 if the kernel aborted (host stopped feeding)
+  unsigned long long* signal; // host-mapped completion counter
+  unsigned long long* span;   // optional: 64 task-start slots (time_kernels)
+  unsigned long long* span_acc;
+  unsigned long long* phase;  // diagnostics (BM_PHASE_DUMP): per-CTA timestamps of task 20
+};
+cudaError_t launch_lstm_persistent(const PersistArgs& a, cudaStream_t st);
+int persistent_smem_bytes();
+
 // bf16 / tcgen05 path (cell_step_sm100.cu). a.W: weights in the stage-tile layout
 // (launch_pack_tiles): [tile][K/64][tile_rows][64] bf16, 128B-swizzled rows.
 cudaError_t launch_cell_step_sm100(const StepArgs& a, cudaStream_t st);

@@ -212,6 +212,35 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
     off += t.b;
   }
   e.ring_head = off;
+  if (e.persistent_active) {
+    // rows first, then the headers that publish them (same copy stream: ordered)
+    CK(cudaMemcpyAsync(e.ring_dev + base, e.ring_host + base, sizeof(RowDesc) * total,
+                       cudaMemcpyHostToDevice, e.copy_stream));
+    const int n = static_cast<int>(tasks.size());
+    const int h0 = static_cast<int>((tasks[0].seq - e.run_base) % e.hdr_ring);
+    for (int i = 0; i < n; ++i) {
+      Task& t = tasks[i];
+      TaskHdr& h = e.hdr_host[(h0 + i) % e.hdr_ring];
+      h.seq = static_cast<int32_t>(t.seq - e.run_base);
+      h.b = t.b;
+      h.row_off = t.ring_off;
+      h.flags = 0;
+      if (e.cfg.time_kernels) {
+        double bytes, flops;
+        algo_cost(e, e.cells[t.ct], t.b, false, &bytes, &flops);
+        e.stats.timed_launches += 1;
+        e.stats.timed_bytes += bytes;
+        e.stats.timed_flops += flops;
+      }
+    }
+    const int first = std::min(n, e.hdr_ring - h0);
+    CK(cudaMemcpyAsync(e.hdr_dev + h0, e.hdr_host + h0, sizeof(TaskHdr) * first, cudaMemcpyHostToDevice,
+                       e.copy_stream));
+    if (first < n)
+      CK(cudaMemcpyAsync(e.hdr_dev, e.hdr_host, sizeof(TaskHdr) * (n - first), cudaMemcpyHostToDevice,
+                         e.copy_stream));
+    return BM_OK;
+  }
   CK(cudaMemcpyAsync(e.ring_dev + base, e.ring_host + base, sizeof(RowDesc) * total,
                      cudaMemcpyHostToDevice, e.stream));
   for (Task& t : tasks) {
@@ -339,6 +368,7 @@ void bm_config_default(bm_config* c) {
   c->record_logits = 0;
   c->time_kernels = 0;
   c->record_log = 1;
+  c->persistent = 0;
 }
 
 static void free_device(Engine& e) {
@@ -373,6 +403,11 @@ static void free_device(Engine& e) {
     cudaEventDestroy(t.end);
   }
   cudaFree(e.spans);
+  if (e.copy_stream) cudaStreamDestroy(e.copy_stream);
+  cudaFree(e.hdr_dev);
+  if (e.hdr_host) cudaFreeHost(e.hdr_host);
+  cudaFree(e.gbar);
+  cudaFree(e.perr);
   if (e.stream) cudaStreamDestroy(e.stream);
 }
 
@@ -693,6 +728,105 @@ bm_status bm_poll(bm_engine* h, bm_completion* out, int cap, int* n) {
   return BM_OK;
 }
 
+static bool persistent_eligible(const Engine& e) {
+  if (!e.cfg.persistent || !e.device() || e.cfg.precision != BM_PREC_BF16 || e.cells.size() != 1) return false;
+  const Cell& c = e.cells[0];
+  const int K = c.K0 + c.K1;
+  return c.d.kind == BM_CELL_LSTM && c.d.layers == 1 && c.S >= 1 && c.S <= 4 && c.kslice <= 512 &&
+         c.kslice % 64 == 0 && e.cfg.hidden % 32 == 0 && c.d.max_batch <= 512 && K == c.S * c.kslice;
+}
+
+static bm_status persistent_start(Engine& e) {
+  const Cell& c = e.cells[0];
+  if (e.copy_stream == nullptr) {
+    CK(cudaStreamCreateWithFlags(&e.copy_stream, cudaStreamNonBlocking));
+    CK(cudaMalloc(&e.hdr_dev, sizeof(TaskHdr) * e.hdr_ring));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&e.hdr_host), sizeof(TaskHdr) * e.hdr_ring, cudaHostAllocDefault));
+    CK(cudaMalloc(&e.gbar, sizeof(unsigned int)));
+    CK(cudaMalloc(&e.perr, sizeof(int)));
+  }
+  CK(cudaStreamSynchronize(e.stream));
+  CK(cudaMemsetAsync(e.hdr_dev, 0xFF, sizeof(TaskHdr) * e.hdr_ring, e.stream));  // seq = -1
+  CK(cudaMemsetAsync(e.gbar, 0, sizeof(unsigned int), e.stream));
+  CK(cudaMemsetAsync(e.perr, 0, sizeof(int), e.stream));
+  PersistArgs a{};
+  a.H = e.cfg.hidden;
+  a.K = c.K0 + c.K1;
+  a.K0 = c.K0;
+  a.S = c.S;
+  a.kslice = c.kslice;
+  a.n_slots = e.cfg.max_slots;
+  a.res_layers = e.cfg.pool_layers;
+  a.hdr_ring = e.hdr_ring;
+  a.hdr = e.hdr_dev;
+  a.rows = e.ring_dev;
+  a.E = c.E;
+  a.h_pool = e.h_layer(0);
+  a.c_pool = e.c_layer(0);
+  a.tok = e.tok;
+  a.W = c.W[0];
+  a.bias = c.bias[0];
+  a.res_h = e.res_h;
+  a.res_c = e.res_c;
+  a.gbar = e.gbar;
+  a.err = e.perr;
+  a.signal = e.signal_dev;
+  a.span = e.cfg.time_kernels ? e.spans : nullptr;
+  a.span_acc = e.cfg.time_kernels ? e.spans + 128 : nullptr;
+  static const char* dump = getenv("BM_PHASE_DUMP");
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 16 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 16 * 4096, e.stream));
+  a.phase = e.phase_dev;
+  cudaError_t err = launch_lstm_persistent(a, e.stream);
+  if (err == cudaErrorCooperativeLaunchTooLarge) {
+    cudaGetLastError();
+    return BM_E_AGAIN;  // cannot co-schedule every CTA: fall back to per-task launches
+  }
+  CK(err);
+  e.persistent_active = true;
+  e.run_base = e.launched;
+  e.stats.kernel_launches += 1;
+  return BM_OK;
+}
+
+static bm_status persistent_stop(Engine& e) {
+  if (!e.persistent_active) return BM_OK;
+  const int idx = static_cast<int>((e.launched - e.run_base) % e.hdr_ring);
+  // the slot's previous task retired long ago (at most k + MaxTasksToSubmit are in flight)
+  TaskHdr& hd = e.hdr_host[idx];
+  hd.seq = static_cast<int32_t>(e.launched - e.run_base);
+  hd.b = -1;
+  hd.row_off = 0;
+  hd.flags = 0;
+  CK(cudaMemcpyAsync(e.hdr_dev + idx, &hd, sizeof(TaskHdr), cudaMemcpyHostToDevice, e.copy_stream));
+  CK(cudaStreamSynchronize(e.copy_stream));
+  CK(cudaStreamSynchronize(e.stream));
+  e.persistent_active = false;
+  static const char* dump = getenv("BM_PHASE_DUMP");
+  if (dump != nullptr && e.phase_dev != nullptr) {
+    std::vector<unsigned long long> hh(16 * 4096);
+    CK(cudaMemcpy(hh.data(), e.phase_dev, hh.size() * 8, cudaMemcpyDeviceToHost));
+    FILE* f = fopen(dump, "a");
+    if (f) {
+      fprintf(f, "persistent task 20\n");
+      for (int i = 0; i < 4096; ++i)
+        if (hh[i * 16]) {
+          fprintf(f, "%d", i);
+          for (int k = 0; k < 16; ++k) fprintf(f, " %llu", hh[i * 16 + k]);
+          fprintf(f, "\n");
+        }
+      fclose(f);
+    }
+  }
+  int aborted = 0;
+  CK(cudaMemcpy(&aborted, e.perr, sizeof(int), cudaMemcpyDeviceToHost));
+  if (aborted) {
+    e.sticky_cuda = true;
+    return BM_E_CUDA;
+  }
+  return BM_OK;
+}
+
 bm_status bm_run(bm_engine* h, int* n_completed) {
   if (h == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
@@ -700,6 +834,11 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
   const size_t before = e.completions.size();
   int n = 0;
   bm_status s = BM_OK;
+  if (persistent_eligible(e)) {
+    s = persistent_start(e);
+    if (s != BM_OK && s != BM_E_AGAIN) return s;
+    s = BM_OK;
+  }
   if (e.cfg.clock == BM_CLOCK_WALL) {
     e.t0 = std::chrono::steady_clock::now();
     e.wall_started = true;
@@ -708,13 +847,23 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
       retire_ready(e, false);
       admit_due(e);
       s = schedule_and_launch(e, &n);
-      if (s != BM_OK) return s;
+      if (s != BM_OK) {
+        persistent_stop(e);
+        return s;
+      }
       if (all_done(e)) break;
     }
   } else {
     while ((s = virtual_round(e, &n)) == BM_OK) {
     }
-    if (s != BM_E_AGAIN) return s;
+    if (s != BM_E_AGAIN) {
+      persistent_stop(e);
+      return s;
+    }
+  }
+  if (e.persistent_active) {
+    s = persistent_stop(e);
+    if (s != BM_OK) return s;
   }
   if (e.device()) CK(cudaStreamSynchronize(e.stream));
   if (n_completed) *n_completed = static_cast<int>(e.completions.size() - before);

@@ -26,14 +26,16 @@ def _check_log(e, rp):
     assert [(c.req_id, c.t_done) for c in comp] == [(rid, float(tk)) for rid, tk in rp.completions]
 
 
+@pytest.mark.parametrize("persistent", [0, 1])
 @pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
 @pytest.mark.parametrize("minf", [1, 4])
-def test_config0_end_to_end(prec, minf):
+def test_config0_end_to_end(prec, minf, persistent):
     """BASELINE configs[0]: 1-layer LSTM, h=64, 4 requests (3, 10, 5, 8), arrivals (0, 0, 1, 3),
-    bmax 4, virtual clock."""
+    bmax 4, virtual clock; also through the persistent weight-stationary kernel (bf16)."""
     trace = gen.config0_trace(vocab=128)
     e, cid, w = lstm_engine(64, 1, 128, prec, bmax=4, clock=bm.CLOCK_VIRTUAL, max_slots=16,
-                            max_requests=16, keep_results=1, min_followon_batch=minf)
+                            max_requests=16, keep_results=1, min_followon_batch=minf,
+                            persistent=persistent)
     for q in trace:
         e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
     e.run()
@@ -46,13 +48,15 @@ def test_config0_end_to_end(prec, minf):
         assert np.max(np.abs(r["c"][0] - cs[0])) <= TOL[prec]
 
 
-@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
-def test_wmt_chain_h1024(prec):
+@pytest.mark.parametrize("prec,persistent", [(bm.PREC_BF16, 0), (bm.PREC_BF16, 1), (bm.PREC_FP32, 0)])
+def test_wmt_chain_h1024(prec, persistent):
     """configs[1] shape at a size the oracle finishes in seconds: 48 WMT-length requests,
-    Poisson arrivals, h=1024, bmax 512, virtual clock with look-ahead k=2."""
+    Poisson arrivals, h=1024, bmax 512, virtual clock with look-ahead k=2; bf16 also through the
+    persistent weight-stationary kernel."""
     trace = gen.chain_trace(48, 2048, seed=1000, rate=2.0)
     e, cid, w = lstm_engine(1024, 1, 2048, prec, bmax=512, clock=bm.CLOCK_VIRTUAL, max_slots=256,
-                            max_requests=256, keep_results=1, schedule_when_outstanding_leq=2)
+                            max_requests=256, keep_results=1, schedule_when_outstanding_leq=2,
+                            persistent=persistent)
     for q in trace:
         e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
     e.run()
@@ -124,12 +128,13 @@ def test_treebank_trees_h1024(prec):
         assert np.max(np.abs(r["c"][0] - rc)) <= TOL[prec]
 
 
-def test_wall_clock_run_completes_and_matches_oracle():
+@pytest.mark.parametrize("persistent", [0, 1])
+def test_wall_clock_run_completes_and_matches_oracle(persistent):
     """The open-loop driver on the wall clock (bench path): all requests complete, results
     match the oracle (scheduling then depends on timing, results must not)."""
     trace = gen.chain_trace(64, 1024, seed=5, rate=20000.0)
     e, cid, w = lstm_engine(1024, 1, 1024, bm.PREC_BF16, bmax=512, max_slots=256, max_requests=256,
-                            keep_results=1, schedule_when_outstanding_leq=2)
+                            keep_results=1, schedule_when_outstanding_leq=2, persistent=persistent)
     for q in trace:
         e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
     assert e.run() == 64
@@ -139,3 +144,25 @@ def test_wall_clock_run_completes_and_matches_oracle():
         r = e.read_result(i, 1)
         hs, cs = cells.chain_lstm(w, trace[i].tokens)
         assert np.max(np.abs(r["h"][0] - hs[0])) <= TOL[bm.PREC_BF16]
+    # a second run on the same engine (the persistent kernel is relaunched per bm_run)
+    for q in trace[:8]:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    assert e.run() == 8
+
+
+def test_persistent_large_batches_match_launch_path():
+    """Persistent kernel with 300-row tasks (3 column chunks) equals the per-task launch path
+    on the same trace (both bf16, results within tolerance of each other and the oracle)."""
+    trace = gen.chain_trace(600, 1024, seed=9, lengths=[3] * 600, arrivals=[0] * 600)
+    res = []
+    for persistent in (0, 1):
+        e, cid, w = lstm_engine(1024, 1, 1024, bm.PREC_BF16, bmax=300, clock=bm.CLOCK_VIRTUAL,
+                                max_slots=1024, max_requests=1024, keep_results=1, persistent=persistent)
+        for q in trace:
+            e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+        assert e.run() == 600
+        res.append(np.stack([e.read_result(i, 1)["h"][0] for i in range(600)]))
+    assert np.max(np.abs(res[0] - res[1])) <= 1e-2
+    for i in (0, 299, 599):
+        hs, _ = cells.chain_lstm(w, trace[i].tokens)
+        assert np.max(np.abs(res[1][i] - hs[0])) <= TOL[bm.PREC_BF16]
