@@ -203,7 +203,8 @@ struct Engine {
   int direct_flip = 0;
   // persistent weight-stationary LSTM (bm_config.persistent)
   bool persistent_active = false;
-  cudaStream_t copy_stream = nullptr;  // ring copies while the persistent kernel owns `stream`
+  cudaStream_t copy_stream = nullptr;  // descriptor-ring copies (off the kernel stream)
+  cudaEvent_t copy_ev = nullptr;
   TaskHdr* hdr_dev = nullptr;
   TaskHdr* hdr_host = nullptr;         // pinned staging
   int hdr_ring = 256;

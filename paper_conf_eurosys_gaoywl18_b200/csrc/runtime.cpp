@@ -241,8 +241,13 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
                          e.copy_stream));
     return BM_OK;
   }
+  // descriptors travel on the copy stream: the copy overlaps the kernels still running, and the
+  // kernel stream only waits on an event that has usually fired by the time it gets there (an
+  // in-stream copy would sit between two launches, on the critical path, and break PDL)
   CK(cudaMemcpyAsync(e.ring_dev + base, e.ring_host + base, sizeof(RowDesc) * total,
-                     cudaMemcpyHostToDevice, e.stream));
+                     cudaMemcpyHostToDevice, e.copy_stream));
+  CK(cudaEventRecord(e.copy_ev, e.copy_stream));
+  CK(cudaStreamWaitEvent(e.stream, e.copy_ev, 0));
   for (Task& t : tasks) {
     bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, t.b, &t, e.signal_dev);
     if (s != BM_OK) return s;
@@ -404,6 +409,7 @@ static void free_device(Engine& e) {
   }
   cudaFree(e.spans);
   if (e.copy_stream) cudaStreamDestroy(e.copy_stream);
+  if (e.copy_ev) cudaEventDestroy(e.copy_ev);
   cudaFree(e.hdr_dev);
   if (e.hdr_host) cudaFreeHost(e.hdr_host);
   cudaFree(e.gbar);
@@ -439,7 +445,10 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
     if (cudaGetDeviceProperties(&prop, c.device) != cudaSuccess || prop.major != 10)
       return fail(BM_E_NODEV);
     if (cudaSetDevice(c.device) != cudaSuccess) return fail(BM_E_NODEV);
-    if (cudaStreamCreateWithFlags(&E.stream, cudaStreamNonBlocking) != cudaSuccess) return fail(BM_E_CUDA);
+    if (cudaStreamCreateWithFlags(&E.stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&E.copy_stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&E.copy_ev, cudaEventDisableTiming) != cudaSuccess)
+      return fail(BM_E_CUDA);
     const size_t H = c.hidden, S = c.max_slots, L = c.pool_layers, R = c.max_requests;
     const size_t el = E.elem();
     bool ok = cudaMalloc(&E.h_pool, L * 2 * S * H * el) == cudaSuccess &&
@@ -738,8 +747,7 @@ static bool persistent_eligible(const Engine& e) {
 
 static bm_status persistent_start(Engine& e) {
   const Cell& c = e.cells[0];
-  if (e.copy_stream == nullptr) {
-    CK(cudaStreamCreateWithFlags(&e.copy_stream, cudaStreamNonBlocking));
+  if (e.hdr_dev == nullptr) {
     CK(cudaMalloc(&e.hdr_dev, sizeof(TaskHdr) * e.hdr_ring));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&e.hdr_host), sizeof(TaskHdr) * e.hdr_ring, cudaHostAllocDefault));
     CK(cudaMalloc(&e.gbar, sizeof(unsigned int)));
