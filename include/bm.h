@@ -258,6 +258,9 @@ typedef struct {
   uint64_t schedule_calls;
   double span_ms;            /* same launches, device-side span (first CTA start .. last  */
                              /* CTA end, %globaltimer): excludes host launch latency      */
+  double launch_ns;          /* host time spent staging descriptors and issuing launches  */
+  double retire_ns;          /* host time spent retiring finished tasks (Retire, A4)      */
+  uint64_t span_launches;    /* launches whose device span is in span_ms                  */
 } bm_stats;
 
 bm_status bm_get_stats(bm_engine* e, bm_stats* out);

@@ -82,7 +82,9 @@ class Stats(C.Structure):
     _fields_ = [("tasks", C.c_uint64), ("rows", C.c_uint64), ("kernel_launches", C.c_uint64),
                 ("timed_launches", C.c_uint64), ("timed_ms", C.c_double),
                 ("timed_bytes", C.c_double), ("timed_flops", C.c_double),
-                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64), ("span_ms", C.c_double)]
+                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64), ("span_ms", C.c_double),
+                ("launch_ns", C.c_double), ("retire_ns", C.c_double),
+                ("span_launches", C.c_uint64)]
 
 
 # exported symbols (tests/test_abi.py checks them against include/bm.h)

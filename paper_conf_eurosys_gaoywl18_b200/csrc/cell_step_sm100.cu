@@ -26,6 +26,7 @@
 // move the accumulators TMEM -> smem, the cluster reduces, and warps 0-7 run the epilogue.
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "kernels.h"
 #include "sm100_ptx.cuh"
@@ -35,7 +36,7 @@ namespace {
 using namespace ptx;
 
 constexpr int kMaxStages = 8;           // pipeline depth cap
-constexpr int kTailBytes = 5120;        // row-source table [2][256] + barriers, at smem offset 0
+constexpr int kTailBytes = 1024;        // barriers + TMEM slot, at smem offset 0
 constexpr int kBK = 64;                 // K elements per stage (128 B of bf16 = one SW128 atom)
 constexpr int kProducerThreads = 256;   // warps 0-7: activation gather (cp.async)
 constexpr int kMmaWarp = 8;             // warp 8: TMEM alloc + tcgen05.mma issue
@@ -59,15 +60,16 @@ constexpr int kWRing = 2;               // weight chunks in the ring
 // Small tasks (npad <= 128) use 32 KB weight chunks and a 32 KB activation ring so the CTA fits
 // in ~100 KB and two CTAs share an SM: under PDL the next launch's weight stream and gather
 // overlap this launch's split-K epilogue. Larger tasks use 64 KB chunks and a 64 KB ring.
+// Default plan; the launcher passes the chosen chunk size / ring size in StepArgs.
 __host__ __device__ __forceinline__ int w_chunk_blocks(int npad) { return npad <= 128 ? 2 : kWChunkMax; }
 __host__ __device__ __forceinline__ int x_ring_bytes(int npad) { return npad <= 128 ? 32 * 1024 : 64 * 1024; }
-__host__ __device__ __forceinline__ int x_stages_for(int npad) {
-  const int n = x_ring_bytes(npad) / (npad * 128);
+__host__ __device__ __forceinline__ int x_stages_for(int npad, int xring) {
+  const int n = xring / (npad * 128);
   return n < 2 ? 2 : (n > kMaxStages ? kMaxStages : n);
 }
 // weight ring + activation ring, reused after the main loop for the partial / logits tile
-__host__ __device__ __forceinline__ int region_bytes(int npad) {
-  const int a = kWRing * w_chunk_blocks(npad) * kWStageBytes + x_stages_for(npad) * npad * 128;
+__host__ __device__ __forceinline__ int region_bytes(int npad, int wcb, int xring) {
+  const int a = kWRing * wcb * kWStageBytes + x_stages_for(npad, xring) * npad * 128;
   const int b = 129 * npad * 4 + 4 * 128 * 4;
   return a > b ? a : b;
 }
@@ -86,7 +88,7 @@ __device__ __forceinline__ void phase_mark(const StepArgs& p, int i) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-    p.phase[cta * 16 + i] = t;
+    p.phase[cta * 32 + i] = t;
   }
 }
 
@@ -138,15 +140,15 @@ __global__ void __launch_bounds__(kThreads, 2)
   const int npad = (ncols + 15) & ~15;
   const int nk = p.kslice / kBK;
   const int k_begin = static_cast<int>(rank) * p.kslice;
-  const int kStages = p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad)) : x_stages_for(npad);
-  const int wcb = w_chunk_blocks(npad);                   // ring slot capacity in K blocks
+  const int kStages = p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad, p.xring))
+                                       : x_stages_for(npad, p.xring);
+  const int wcb = p.wcb;                                  // ring slot capacity in K blocks
   const int kpc = min(wcb, nk);                           // K blocks per weight chunk
   const int n_chunks = (nk + kpc - 1) / kpc;
   const int wblk_bytes = tile_rows * 128;                 // one K block of this CTA's weight tile
 
   // shared memory: [tail: row sources + barriers][weight ring | activation ring]
-  const __nv_bfloat16** src_tab = reinterpret_cast<const __nv_bfloat16**>(base);  // [2][256]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(base + 2 * kMaxCols * sizeof(void*));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(base);
   const uint32_t full0 = smem_u32(bars);                            // activation stage full
   const uint32_t empty0 = smem_u32(bars + kMaxStages);              // activation stage free
   const uint32_t wfull0 = smem_u32(bars + 2 * kMaxStages);          // weight chunk landed
@@ -154,17 +156,18 @@ __global__ void __launch_bounds__(kThreads, 2)
   const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages + 2 * kWRing);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 2 * kWRing + 1);
   int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
-  uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
+  uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 1 KB)
   uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
   uint8_t* x_st = smem + kWRing * wcb * kWStageBytes;     // kStages x npad x 128 B
   const int x_stage_bytes = npad * 128;
 
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
-  if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 16 + 14] = clock64();
+  if (tid == 0 && p.tl != nullptr) atomicMax(p.tl, ~gtimer());
+  if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 32 + 14] = clock64();
   if (tid == 0) {
     for (int s = 0; s < kMaxStages; ++s) {
-      mbar_init(full0 + 8 * s, 1);  // one gather thread arrives after a producer-wide barrier
+      mbar_init(full0 + 8 * s, kProducerThreads);  // every gather thread's cp.async arrive
       mbar_init(empty0 + 8 * s, 1);
     }
     for (int s = 0; s < kWRing; ++s) {
@@ -193,25 +196,44 @@ __global__ void __launch_bounds__(kThreads, 2)
     pdl_wait();  // rows, pool h/c and feed tokens are written by earlier launches / copies
     // device span starts when the launch's dependent work may begin (after the PDL wait)
     if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
+    if (tid == 0 && p.tl != nullptr) atomicMax(p.tl + 1, ~gtimer());
     if (tid == 0) phase_mark(p, 8);
-    for (int c = tid; c < kMaxCols; c += kProducerThreads) {
-      const __nv_bfloat16* s0 = nullptr;
-      const __nv_bfloat16* s1 = nullptr;
-      if (c < ncols) {
-        const RowDesc r = p.rows[col0 + c];
-        s0 = seg_src<EPI>(p, r, 0);
-        if (p.K1 > 0) s1 = seg_src<EPI>(p, r, 1);
-      }
-      src_tab[c] = s0;
-      src_tab[kMaxCols + c] = s1;
+    // Each producer thread owns fixed (row, 16-B chunk) items of every stage: item q = tid +
+    // 256 i, row = q / 8, chunk = q % 8 (8 threads cover a row's 128-B K block, coalesced).
+    // Row sources are resolved once into registers (no per-stage table lookups).
+    constexpr int kItems = kMaxCols * 8 / kProducerThreads;  // 8
+    const int n_items = (npad * 8 + kProducerThreads - 1 - tid) / kProducerThreads;
+    const __nv_bfloat16* src0[kItems];
+    const __nv_bfloat16* src1[kItems];
+    uint32_t dst_off[kItems];
+    RowDesc rd[kItems];
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {  // independent loads first (clamped, unconditional)
+      const int row = min((tid + i * kProducerThreads) >> 3, ncols - 1);
+      const int4 v = __ldg(reinterpret_cast<const int4*>(p.rows) + col0 + row);
+      rd[i] = RowDesc{v.x, v.y, v.z, v.w};
     }
-    named_bar(1, kProducerThreads);
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {
+      const int q = tid + i * kProducerThreads;
+      const int row = q >> 3;
+      const int ch = q & 7;
+      dst_off[i] = row * 128 + ((ch ^ (row & 7)) << 4);
+      src0[i] = nullptr;
+      src1[i] = nullptr;
+      if (i < n_items && row < ncols) {
+        const __nv_bfloat16* a0 = seg_src<EPI>(p, rd[i], 0);
+        const __nv_bfloat16* a1 = p.K1 > 0 ? seg_src<EPI>(p, rd[i], 1) : nullptr;
+        src0[i] = a0 != nullptr ? a0 + ch * 8 : nullptr;
+        src1[i] = a1 != nullptr ? a1 + ch * 8 : nullptr;
+      }
+    }
     if (tid == 0) phase_mark(p, 9);
-    // Every stage's cp.async group stays in flight until the ring is full; a stage is handed
-    // to the MMA (full barrier) once its group has landed and been made visible to the
-    // async proxy. lag = stages - 1 keeps the whole ring in flight without deadlock.
+    // A stage is handed to the MMA by the hardware: every producer thread's
+    // cp.async.mbarrier.arrive.noinc fires once that thread's copies of the stage have landed
+    // (full barrier count = 256), so no producer waits on its own copies.
     const __nv_bfloat16* dummy = static_cast<const __nv_bfloat16*>(p.E != nullptr ? p.E : p.h_pool);
-    const int lag = min(kStages - 1, 7);
+    const bool no_reads = (p.experiment & 1) != 0;
     for (int kb = 0; kb < nk; ++kb) {
       const int s = kb % kStages;
       const int round = kb / kStages;
@@ -220,40 +242,24 @@ __global__ void __launch_bounds__(kThreads, 2)
       const int seg = k >= p.K0 ? 1 : 0;
       const int kk = k - seg * p.K0;
       const uint32_t xs = smem_u32(x_st + s * x_stage_bytes);
-      const __nv_bfloat16** tab = src_tab + seg * kMaxCols;
       if (p.experiment & 4) {  // diagnostics: no gather at all, hand the stage over at once
-        if (tid == 0) mbar_arrive(full0 + 8 * s);
+        mbar_arrive(full0 + 8 * s);
         continue;
       }
-      for (int q = tid; q < npad * 8; q += kProducerThreads) {
-        const int row = q >> 3;
-        const int ch = q & 7;
-        const __nv_bfloat16* src = (p.experiment & 1) ? nullptr : tab[row];
-        const uint32_t dst = xs + row * 128 + ((ch ^ (row & 7)) << 4);
-        if (src != nullptr) {
-          cp_async_16(dst, src + kk + ch * 8, 16);
-        } else {
-          cp_async_16(dst, dummy, 0);  // zero fill
+#pragma unroll
+      for (int i = 0; i < kItems; ++i) {
+        if (i < n_items) {
+          const __nv_bfloat16* src = seg ? src1[i] : src0[i];
+          if (src != nullptr && !no_reads) {
+            cp_async_16(xs + dst_off[i], src + kk, 16);
+          } else {
+            cp_async_16(xs + dst_off[i], dummy, 0);  // zero fill
+          }
         }
       }
-      cp_async_commit();
+      cp_async_arrive_noinc(full0 + 8 * s);
       if (tid == 0 && kb == 0) phase_mark(p, 10);
-      if (kb >= lag) {
-        // every producer's copies of stage kb - lag have landed and are visible to the async
-        // proxy; one thread then hands the stage to the MMA (256 release-arrives per stage
-        // measured ~0.3 us per hand-off, a named barrier + one arrive ~0.05 us)
-        cp_async_wait_dyn(lag);
-        fence_proxy_async();
-        named_bar(1, kProducerThreads);
-        if (tid == 0 && kb == lag) phase_mark(p, 11);
-        if (tid == 0) mbar_arrive(full0 + 8 * ((kb - lag) % kStages));
-      }
     }
-    cp_async_wait<0>();
-    fence_proxy_async();
-    named_bar(1, kProducerThreads);
-    if (!(p.experiment & 4) && tid == 0)
-      for (int kb = max(0, nk - lag); kb < nk; ++kb) mbar_arrive(full0 + 8 * (kb % kStages));
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
     // Weights are read-only: streaming starts before griddepcontrol.wait (PDL overlap).
@@ -295,6 +301,8 @@ __global__ void __launch_bounds__(kThreads, 2)
       if (lane == 0 && kb == 0) phase_mark(p, 6);
       if (lane == 0 && kb == nk - 1) phase_mark(p, 7);
       if (lane == 0 && kb == 1) phase_mark(p, 12);
+      if (lane == 0 && kb < 12) phase_mark(p, 16 + kb);   // stage kb at the MMA
+      if (lane == 0 && kb % kpc == 0 && c < 4) phase_mark(p, 28 + c);  // weight chunk c at the MMA
       if (lane == 0) {
         const uint64_t a =
             sdesc_sw128(smem_u32(w_ring + ws * wcb * kWStageBytes + (kb % kpc) * wblk_bytes));
@@ -486,7 +494,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (tid == 0) phase_mark(p, 4);
     cluster_sync();  // B: peers may read this CTA's partials until here
     if (tid == 0) phase_mark(p, 5);
-    if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 16 + 15] = clock64();
+    if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 32 + 15] = clock64();
     if (p.signal != nullptr) {  // completion signal (A12) fused into the task's last CTA
       __threadfence();
       __syncthreads();
@@ -506,6 +514,13 @@ __global__ void __launch_bounds__(kThreads, 2)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256)
                  : "memory");
   }
+  if (p.tl != nullptr) {
+    __syncthreads();
+    if (tid == 0) {
+      atomicMax(p.tl + 2, gtimer());
+      atomicAdd(p.tl + 3, 1ull);
+    }
+  }
   if (p.span != nullptr) {  // device-side span: first CTA start .. last CTA end
     __syncthreads();
     if (tid == 0) {
@@ -522,20 +537,23 @@ __global__ void __launch_bounds__(kThreads, 2)
 }
 
 template <int EPI>
-cudaError_t launch_impl(const StepArgs& a, cudaStream_t st) {
+cudaError_t launch_impl(StepArgs a, cudaStream_t st) {
   static bool configured = false;
   if (!configured) {
-    const int max_smem = 1024 + kTailBytes + region_bytes(16) > 1024 + kTailBytes + region_bytes(kMaxCols)
-                             ? 1024 + kTailBytes + region_bytes(16)
-                             : 1024 + kTailBytes + region_bytes(kMaxCols);
     cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, max_smem);
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     if (e != cudaSuccess) return e;
     configured = true;
   }
   const int cols = a.b < kMaxCols ? a.b : kMaxCols;
   const int npad = (cols + 15) & ~15;
-  const size_t smem = 1024 + kTailBytes + region_bytes(npad);
+  // ring plan (BM_WCB = K blocks per weight chunk, BM_XRING = activation ring KB: experiments)
+  static const int env_wcb = getenv("BM_WCB") ? atoi(getenv("BM_WCB")) : 0;
+  static const int env_xring = getenv("BM_XRING") ? atoi(getenv("BM_XRING")) : 0;
+  a.wcb = env_wcb > 0 ? env_wcb : w_chunk_blocks(npad);
+  a.xring = env_xring > 0 ? env_xring * 1024 : x_ring_bytes(npad);
+  const size_t smem = 1024 + kTailBytes + region_bytes(npad, a.wcb, a.xring);
+  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int S = EPI == EPI_PROJ ? 1 : a.S;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;
   cudaLaunchConfig_t cfg = {};

@@ -216,6 +216,13 @@ struct Engine {
   unsigned long long* spans = nullptr;  // device: 64 span slots + accumulator (time_kernels)
   unsigned long long span_base[2] = {0, 0};
   uint64_t launches_base = 0;
+  // diagnostics (BM_TIMELINE=<file>): per-launch device times + host issue times, per-task
+  // host retire times; written at bm_destroy
+  static constexpr uint64_t kTimeline = 8192;
+  unsigned long long* tl_dev = nullptr;
+  std::vector<long long> tl_host, tl_retire;
+  std::vector<int> tl_b;
+  uint64_t tl_n = 0;
 
   bool device() const { return cfg.clock != BM_CLOCK_DRY; }
   size_t elem() const { return cfg.precision == BM_PREC_BF16 ? 2 : 4; }

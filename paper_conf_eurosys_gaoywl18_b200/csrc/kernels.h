@@ -64,8 +64,12 @@ struct StepArgs {
   unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
   unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)
   int pdl;                    // launch with programmatic dependent launch (overlap setup)
+  int wcb, xring;             // ring plan (set by the launcher): K blocks per weight chunk,
+                              // activation ring bytes
   unsigned long long* span;   // time_kernels: slot {min CTA start, CTAs done} (device memory)
   unsigned long long* span_acc;  // {sum of launch spans in ns, launches}: last CTA adds
+  unsigned long long* tl;     // diagnostics (BM_TIMELINE): {~first CTA start, ~first past the
+                              // PDL wait, last CTA end, CTAs} in %globaltimer ns, or null
 };
 
 // Persistent weight-stationary LSTM engine (lstm_persistent_sm100.cu).

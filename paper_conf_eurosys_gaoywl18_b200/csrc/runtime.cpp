@@ -20,6 +20,12 @@
 
 namespace bm {
 
+long long realtime_ns() {
+  timespec ts;
+  clock_gettime(CLOCK_REALTIME, &ts);
+  return static_cast<long long>(ts.tv_sec) * 1000000000LL + ts.tv_nsec;
+}
+
 double wall_now(const Engine& e) {
   return std::chrono::duration<double>(std::chrono::steady_clock::now() - e.t0).count();
 }
@@ -129,6 +135,12 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
     a.span_acc = e.spans + 128;
     CK(cudaEventRecord(tl->beg, e.stream));
     if (ev_out) *ev_out = i;
+  }
+  if (e.tl_dev != nullptr && e.tl_n < Engine::kTimeline) {
+    a.tl = e.tl_dev + 4 * e.tl_n;
+    e.tl_host[e.tl_n] = realtime_ns();
+    e.tl_b[e.tl_n] = b;
+    e.tl_n += 1;
   }
   cudaError_t err;
   if (e.cfg.precision == BM_PREC_BF16) {
@@ -270,7 +282,9 @@ static int retire_ready(Engine& e, bool block) {
         }
       }
     }
+    if (e.tl_dev != nullptr && t.seq < Engine::kTimeline) e.tl_retire[t.seq] = realtime_ns();
     if (e.cfg.clock == BM_CLOCK_WALL) e.now = wall_now(e);
+    const auto t0 = std::chrono::steady_clock::now();
     retire_task(e, t);
     if (t.ev_count > 0) {
       for (int k = 0; k < t.ev_count; ++k) {
@@ -285,6 +299,7 @@ static int retire_ready(Engine& e, bool block) {
       }
     }
     e.inflight.pop_front();
+    e.stats.retire_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
     ++n;
   }
   return n;
@@ -308,7 +323,9 @@ static bm_status schedule_and_launch(Engine& e, int* n_tasks) {
   e.stats.sched_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
   e.stats.schedule_calls += 1;
   if (tasks.empty()) return BM_OK;
+  const auto t1 = std::chrono::steady_clock::now();
   bm_status s = launch_tasks(e, tasks);
+  e.stats.launch_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t1).count();
   if (s != BM_OK) return s;
   for (Task& t : tasks) e.inflight.push_back(std::move(t));
   *n_tasks = static_cast<int>(tasks.size());
@@ -376,8 +393,26 @@ void bm_config_default(bm_config* c) {
   c->persistent = 0;
 }
 
+static void dump_timeline(Engine& e) {
+  const char* path = getenv("BM_TIMELINE");
+  if (path == nullptr || e.tl_dev == nullptr || cudaStreamSynchronize(e.stream) != cudaSuccess) return;
+  std::vector<unsigned long long> d(4 * Engine::kTimeline);
+  if (cudaMemcpy(d.data(), e.tl_dev, d.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return;
+  FILE* f = fopen(path, "a");
+  if (f == nullptr) return;
+  fprintf(f, "# launch b host_issue_ns dev_start_ns dev_wait_ns dev_end_ns ctas\n");
+  for (uint64_t i = 0; i < e.tl_n; ++i)
+    fprintf(f, "L %llu %d %lld %llu %llu %llu %llu\n", static_cast<unsigned long long>(i), e.tl_b[i],
+            e.tl_host[i], ~d[4 * i], ~d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+  for (uint64_t i = 0; i < std::min<uint64_t>(e.launched, Engine::kTimeline); ++i)
+    if (e.tl_retire[i]) fprintf(f, "R %llu %lld\n", static_cast<unsigned long long>(i), e.tl_retire[i]);
+  fclose(f);
+}
+
 static void free_device(Engine& e) {
   if (!e.device()) return;
+  dump_timeline(e);
+  cudaFree(e.tl_dev);
   for (Cell& c : e.cells) {
     for (void* p : c.W) cudaFree(p);
     for (float* p : c.bias) cudaFree(p);
@@ -493,6 +528,14 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
         if (cudaEventCreate(&t.beg) != cudaSuccess || cudaEventCreate(&t.end) != cudaSuccess)
           return fail(BM_E_CUDA);
       }
+    }
+    if (getenv("BM_TIMELINE") != nullptr) {
+      if (dalloc(&E.tl_dev, 4 * Engine::kTimeline) != cudaSuccess ||
+          cudaMemsetAsync(E.tl_dev, 0, 4 * Engine::kTimeline * 8, E.stream) != cudaSuccess)
+        return fail(BM_E_NOMEM);
+      E.tl_host.assign(Engine::kTimeline, 0);
+      E.tl_retire.assign(Engine::kTimeline, 0);
+      E.tl_b.assign(Engine::kTimeline, 0);
     }
     if (cudaStreamSynchronize(E.stream) != cudaSuccess) return fail(BM_E_CUDA);
   }
@@ -782,8 +825,8 @@ static bm_status persistent_start(Engine& e) {
   a.span = e.cfg.time_kernels ? e.spans : nullptr;
   a.span_acc = e.cfg.time_kernels ? e.spans + 128 : nullptr;
   static const char* dump = getenv("BM_PHASE_DUMP");
-  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 16 * 4096));
-  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 16 * 4096, e.stream));
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 32 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 32 * 4096, e.stream));
   a.phase = e.phase_dev;
   cudaError_t err = launch_lstm_persistent(a, e.stream);
   if (err == cudaErrorCooperativeLaunchTooLarge) {
@@ -997,21 +1040,21 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
   }
   // diagnostics: BM_PHASE_DUMP=<file> records per-CTA phase timestamps of every direct step
   static const char* dump = getenv("BM_PHASE_DUMP");
-  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 16 * 4096));
-  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 16 * 4096, e.stream));
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 32 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 32 * 4096, e.stream));
   bm_status s = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
   if (s != BM_OK) return s;
   if (!async || e.phase_dev) CK(cudaStreamSynchronize(e.stream));
   if (e.phase_dev) {
-    std::vector<unsigned long long> h(16 * 4096);
+    std::vector<unsigned long long> h(32 * 4096);
     CK(cudaMemcpy(h.data(), e.phase_dev, h.size() * 8, cudaMemcpyDeviceToHost));
     FILE* f = fopen(dump, "a");
     if (f) {
       fprintf(f, "step b=%d cell=%d\n", b, cell_id);
       for (int i = 0; i < 4096; ++i)
-        if (h[i * 16]) {
+        if (h[i * 32]) {
           fprintf(f, "%d", i);
-          for (int k = 0; k < 16; ++k) fprintf(f, " %llu", h[i * 16 + k]);
+          for (int k = 0; k < 32; ++k) fprintf(f, " %llu", h[i * 32 + k]);
           fprintf(f, "\n");
         }
       fclose(f);
@@ -1107,6 +1150,7 @@ bm_status bm_get_stats(bm_engine* h, bm_stats* out) {
     CK(cudaStreamSynchronize(e.stream));
     CK(cudaMemcpy(acc, e.spans + 128, 16, cudaMemcpyDeviceToHost));
     out->span_ms = (acc[0] - e.span_base[0]) * 1e-6;
+    out->span_launches = acc[1] - e.span_base[1];
   }
   return BM_OK;
 }

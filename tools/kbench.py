@@ -68,7 +68,8 @@ def main():
         st = e.stats()
         reps = int(os.environ.get("BM_REPEAT", "1"))
         launches = a.iters * reps * (2 if a.cell == "proj" else 1)
-        span_us = st["span_ms"] * 1e3 / launches       # device: first CTA start .. last CTA end
+        # device: first CTA past the PDL wait .. last CTA end, over the sampled launches
+        span_us = st["span_ms"] * 1e3 / max(1, st["span_launches"])
         if a.cell == "proj":
             # LSTM layer + projection per call; report the sum
             byts = (rows_w * K * el + b * 14336) + (V * H * el + b * (2 * H + 8))

@@ -13,7 +13,7 @@ for line in open(sys.argv[1]):
         steps.append(cur)
     else:
         v = [int(x) for x in line.split()]
-        cur["rows"].append(v[1:17])
+        cur["rows"].append(v[1:33] + [0] * (33 - len(v)))
 for st in steps[-3:]:
     a = np.array(st["rows"], dtype=np.float64)
     t0 = a[:, 0].min()
@@ -29,6 +29,11 @@ for st in steps[-3:]:
                   (6, "first stage at MMA (from setup)"), (7, "last stage at MMA (from setup)")):
         d = (a[:, k] - a[:, 1]) / 1e3
         print("  %-32s us: min %.2f med %.2f max %.2f" % (nm, d.min(), np.median(d), d.max()))
+    if a.shape[1] >= 32 and a[:, 16].any():
+        st = [np.median(a[:, 16 + k] - a[:, 1]) / 1e3 for k in range(12) if a[:, 16 + k].all()]
+        wc = [np.median(a[:, 28 + k] - a[:, 1]) / 1e3 for k in range(4) if a[:, 28 + k].all()]
+        print("  stage kb at MMA (med, from setup) us: " + " ".join("%.2f" % x for x in st))
+        print("  weight chunk at MMA (med, from setup) us: " + " ".join("%.2f" % x for x in wc))
     cyc = a[:, 15] - a[:, 14]
     ns = a[:, 5] - a[:, 0]
     ok = (cyc > 0) & (ns > 0)
