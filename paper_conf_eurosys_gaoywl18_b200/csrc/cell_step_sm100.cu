@@ -88,7 +88,7 @@ __device__ __forceinline__ void phase_mark(const StepArgs& p, int i) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-    p.phase[cta * 32 + i] = t;
+    p.phase[cta * 64 + i] = t;
   }
 }
 
@@ -164,7 +164,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
   if (tid == 0 && p.tl != nullptr) atomicMax(p.tl, ~gtimer());
-  if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 32 + 14] = clock64();
+  if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 64 + 14] = clock64();
   if (tid == 0) {
     for (int s = 0; s < kMaxStages; ++s) {
       mbar_init(full0 + 8 * s, kProducerThreads);  // every gather thread's cp.async arrive
@@ -406,13 +406,19 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int cper = (ncols + S - 1) / S;
     float* P = reinterpret_cast<float*>(smem);
     constexpr int pitch = 128;
+    // P row of tile row n = u * G + g: gates padded to Gp = 4 (G <= 4) or 8 (G = 5) floats per
+    // unit, so a unit's gate values are one (or two) aligned 16-byte vector(s) for the reduction
+    constexpr int Gp = (EPI == EPI_INTERNAL) ? 8 : 4;
+    const int prow = (trow / G) * Gp + trow % G;
     if (warp < 8) {
       for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
         float v[32];
         tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
+        if (trow < tile_rows) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i)
-          if (c0 + i < npad) P[(c0 + i) * pitch + trow] = v[i];
+          for (int i = 0; i < 32; ++i)
+            if (c0 + i < npad) P[(c0 + i) * pitch + prow] = v[i];
+        }
       }
     }
     tc_fence_before();
@@ -434,50 +440,49 @@ __global__ void __launch_bounds__(kThreads, 2)
 #pragma unroll
       for (int g = 0; g < 5; ++g) bias[g] = g < G ? p.bias[prow0 + j * G + g] : 0.f;
       for (int cl = tid / U; cl < my_cols; cl += cols_per_pass) {
+        if (tid == 0 && cl / cols_per_pass < 16) phase_mark(p, 32 + cl / cols_per_pass);
         float z[5];
 #pragma unroll
         for (int g = 0; g < 5; ++g) z[g] = bias[g];
-        const uint32_t off = static_cast<uint32_t>(((c_lo + cl) * pitch + j * G) * 4);
+        const uint32_t off = static_cast<uint32_t>(((c_lo + cl) * pitch + j * Gp) * 4);
         // issue every remote load of this item before using any, then add in fixed order
-        if (G == 4) {
-          float4 v[kMaxS];
+        float4 v[kMaxS], w[kMaxS];
+        const bool no_dsmem = (p.experiment & 32) != 0;  // diagnostics: own partial only
 #pragma unroll
-          for (int s = 0; s < kMaxS; ++s)
-            if (s < S) v[s] = ld_cluster_v4(peer[s] + off);
+        for (int s = 0; s < kMaxS; ++s)
+          if (s < S) {
+            const uint32_t a = no_dsmem ? smem_u32(P) + off : peer[s] + off;
+            v[s] = ld_cluster_v4(a);
+            if (G == 5) w[s] = ld_cluster_v4(a + 16);
+          }
 #pragma unroll
-          for (int s = 0; s < kMaxS; ++s)
-            if (s < S) {
-              z[0] += v[s].x;
-              z[1] += v[s].y;
-              z[2] += v[s].z;
-              z[3] += v[s].w;
-            }
+        for (int s = 0; s < kMaxS; ++s)
+          if (s < S) {
+            z[0] += v[s].x;
+            z[1] += v[s].y;
+            z[2] += v[s].z;
+            if (G >= 4) z[3] += v[s].w;
+            if (G == 5) z[4] += w[s].x;
+          }
+        RowDesc r;
+        if (p.experiment & 16) {  // diagnostics: no row / cell-state loads (garbage results)
+          r = RowDesc{0, 0, (c_lo + cl) & 1023, 0};
         } else {
-          float v[kMaxS][5];
-#pragma unroll
-          for (int s = 0; s < kMaxS; ++s)
-#pragma unroll
-            for (int g = 0; g < 5; ++g)
-              if (s < S && g < G) v[s][g] = ld_cluster_f32(peer[s] + off + 4 * g);
-#pragma unroll
-          for (int s = 0; s < kMaxS; ++s)
-#pragma unroll
-            for (int g = 0; g < 5; ++g)
-              if (s < S && g < G) z[g] += v[s][g];
+          const int4 rv = __ldg(reinterpret_cast<const int4*>(p.rows) + col0 + c_lo + cl);
+          r = RowDesc{rv.x, rv.y, rv.z, rv.w};
         }
-        const RowDesc r = p.rows[col0 + c_lo + cl];
         const int u = unit0 + j;
         float hn, cn;
         if constexpr (EPI == EPI_LSTM) {
-          const float cp = (r.flags & ROW_FIRST) ? 0.f : p.c_pool[r.slot * H + u];
+          const float cp = ((r.flags & ROW_FIRST) || (p.experiment & 16)) ? 0.f : p.c_pool[r.slot * H + u];
           cn = sigm(z[1]) * cp + sigm(z[0]) * tanhf(z[2]);
           hn = sigm(z[3]) * tanhf(cn);
         } else if constexpr (EPI == EPI_LEAF) {
           cn = sigm(z[0]) * tanhf(z[2]);
           hn = sigm(z[1]) * tanhf(cn);
         } else {
-          const float cl_ = p.c_pool[static_cast<size_t>(r.a) * H + u];
-          const float cr_ = p.c_pool[static_cast<size_t>(r.b) * H + u];
+          const float cl_ = (p.experiment & 16) ? 0.f : p.c_pool[static_cast<size_t>(r.a) * H + u];
+          const float cr_ = (p.experiment & 16) ? 0.f : p.c_pool[static_cast<size_t>(r.b) * H + u];
           cn = sigm(z[0]) * tanhf(z[4]) + sigm(z[1]) * cl_ + sigm(z[2]) * cr_;
           hn = sigm(z[3]) * tanhf(cn);
         }
@@ -494,7 +499,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (tid == 0) phase_mark(p, 4);
     cluster_sync();  // B: peers may read this CTA's partials until here
     if (tid == 0) phase_mark(p, 5);
-    if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 32 + 15] = clock64();
+    if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 64 + 15] = clock64();
     if (p.signal != nullptr) {  // completion signal (A12) fused into the task's last CTA
       __threadfence();
       __syncthreads();

@@ -825,8 +825,8 @@ static bm_status persistent_start(Engine& e) {
   a.span = e.cfg.time_kernels ? e.spans : nullptr;
   a.span_acc = e.cfg.time_kernels ? e.spans + 128 : nullptr;
   static const char* dump = getenv("BM_PHASE_DUMP");
-  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 32 * 4096));
-  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 32 * 4096, e.stream));
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 64 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 64 * 4096, e.stream));
   a.phase = e.phase_dev;
   cudaError_t err = launch_lstm_persistent(a, e.stream);
   if (err == cudaErrorCooperativeLaunchTooLarge) {
@@ -1040,21 +1040,21 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
   }
   // diagnostics: BM_PHASE_DUMP=<file> records per-CTA phase timestamps of every direct step
   static const char* dump = getenv("BM_PHASE_DUMP");
-  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 32 * 4096));
-  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 32 * 4096, e.stream));
+  if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 64 * 4096));
+  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 64 * 4096, e.stream));
   bm_status s = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
   if (s != BM_OK) return s;
   if (!async || e.phase_dev) CK(cudaStreamSynchronize(e.stream));
   if (e.phase_dev) {
-    std::vector<unsigned long long> h(32 * 4096);
+    std::vector<unsigned long long> h(64 * 4096);
     CK(cudaMemcpy(h.data(), e.phase_dev, h.size() * 8, cudaMemcpyDeviceToHost));
     FILE* f = fopen(dump, "a");
     if (f) {
       fprintf(f, "step b=%d cell=%d\n", b, cell_id);
       for (int i = 0; i < 4096; ++i)
-        if (h[i * 32]) {
+        if (h[i * 64]) {
           fprintf(f, "%d", i);
-          for (int k = 0; k < 32; ++k) fprintf(f, " %llu", h[i * 32 + k]);
+          for (int k = 0; k < 64; ++k) fprintf(f, " %llu", h[i * 64 + k]);
           fprintf(f, "\n");
         }
       fclose(f);

@@ -13,7 +13,7 @@ for line in open(sys.argv[1]):
         steps.append(cur)
     else:
         v = [int(x) for x in line.split()]
-        cur["rows"].append(v[1:33] + [0] * (33 - len(v)))
+        cur["rows"].append(v[1:65] + [0] * (65 - len(v)))
 for st in steps[-3:]:
     a = np.array(st["rows"], dtype=np.float64)
     t0 = a[:, 0].min()
@@ -34,6 +34,9 @@ for st in steps[-3:]:
         wc = [np.median(a[:, 28 + k] - a[:, 1]) / 1e3 for k in range(4) if a[:, 28 + k].all()]
         print("  stage kb at MMA (med, from setup) us: " + " ".join("%.2f" % x for x in st))
         print("  weight chunk at MMA (med, from setup) us: " + " ".join("%.2f" % x for x in wc))
+    if a.shape[1] >= 48 and a[:, 32].any():
+        rp = [np.median(a[:, 32 + k] - a[:, 3]) / 1e3 for k in range(16) if a[:, 32 + k].all()]
+        print("  reduce pass k start (med, from bar1 end) us: " + " ".join("%.2f" % x for x in rp))
     cyc = a[:, 15] - a[:, 14]
     ns = a[:, 5] - a[:, 0]
     ok = (cyc > 0) & (ns > 0)
