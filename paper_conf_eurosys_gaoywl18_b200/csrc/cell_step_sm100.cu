@@ -27,6 +27,7 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 #include <stdlib.h>
+#include <string.h>
 
 #include "kernels.h"
 #include "sm100_ptx.cuh"
@@ -92,7 +93,58 @@ __device__ __forceinline__ void phase_mark(const StepArgs& p, int i) {
   }
 }
 
+// ------------------------------------------------------------------ launch chain
+// Consecutive launches on the engine stream form a chain: the last CTA of launch n publishes
+// n in *dep_flag (release) once every CTA's writes are done; launch n+1, started early under
+// PDL, waits for it with an acquire poll instead of griddepcontrol.wait (grid-completion
+// propagation measured ~3.5 us end -> release on B200; a flag hand-off is a few hundred ns).
+// A poll that has not succeeded after 10 s traps (sticky launch error) instead of hanging.
+__device__ __forceinline__ void dep_wait(const StepArgs& p) {
+  if (p.dep_flag == nullptr) {
+    pdl_wait();
+    return;
+  }
+  const unsigned int want = p.dep_seq - 1u;
+  if ((threadIdx.x & 31) == 0) {
+    unsigned long long t0 = 0;
+    while (static_cast<int>(ld_acquire_gpu(p.dep_flag) - want) < 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 10000000000ull) __trap();
+    }
+  }
+  __syncwarp();
+  (void)ld_acquire_gpu(p.dep_flag);  // every lane acquires the predecessors' writes
+}
+
+// End of a launch: count this CTA; the last one resets the counter, publishes the launch in
+// the chain flag and, on a task's last launch, bumps the host-mapped completion counter (A12).
+__device__ __forceinline__ void launch_done(const StepArgs& p, unsigned int* ctas) {
+  if (threadIdx.x != 0) return;
+  const unsigned total = gridDim.x * gridDim.y * gridDim.z;
+  __threadfence();
+  if (atomicAdd(ctas, 1u) == total - 1) {
+    *ctas = 0;
+    __threadfence();
+    if (p.dep_flag != nullptr) st_release_gpu(p.dep_flag, p.dep_seq);
+    if (p.signal != nullptr) {
+      __threadfence_system();
+      atomicAdd_system(p.signal, 1ull);
+    }
+  }
+}
+
 // ------------------------------------------------------------------ row sources (A6)
+// Row i of the launch: from the inline parameter block, or from device memory (a.rows).
+__device__ __forceinline__ RowDesc row_at(const StepArgs& p, const StepRows& rr, int i) {
+  if (p.rows != nullptr) {
+    const int4 v = __ldg(reinterpret_cast<const int4*>(p.rows) + i);
+    return RowDesc{v.x, v.y, v.z, v.w};
+  }
+  return rr.r[i];
+}
+
 // Pointer to the first element of a row's operand segment `seg`, or nullptr for a zero row.
 template <int EPI>
 __device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const RowDesc& r,
@@ -124,7 +176,7 @@ __device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const
 // ------------------------------------------------------------------ the kernel
 template <int EPI>
 __global__ void __launch_bounds__(kThreads, 2)
-    cell_step_sm100_kernel(const __grid_constant__ StepArgs p) {
+    cell_step_sm100_kernel(const __grid_constant__ StepArgs p, const __grid_constant__ StepRows rr) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
@@ -193,11 +245,7 @@ __global__ void __launch_bounds__(kThreads, 2)
 
   if (warp < 8) {
     // ================================================================ activation gather (A6)
-    pdl_wait();  // rows, pool h/c and feed tokens are written by earlier launches / copies
-    // device span starts when the launch's dependent work may begin (after the PDL wait)
-    if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
-    if (tid == 0 && p.tl != nullptr) atomicMax(p.tl + 1, ~gtimer());
-    if (tid == 0) phase_mark(p, 8);
+
     // Each producer thread owns fixed (row, 16-B chunk) items of every stage: item q = tid +
     // 256 i, row = q / 8, chunk = q % 8 (8 threads cover a row's 128-B K block, coalesced).
     // Row sources are resolved once into registers (no per-stage table lookups).
@@ -208,11 +256,15 @@ __global__ void __launch_bounds__(kThreads, 2)
     uint32_t dst_off[kItems];
     RowDesc rd[kItems];
 #pragma unroll
-    for (int i = 0; i < kItems; ++i) {  // independent loads first (clamped, unconditional)
+    for (int i = 0; i < kItems; ++i) {  // the launch's own rows: independent of earlier launches
       const int row = min((tid + i * kProducerThreads) >> 3, ncols - 1);
-      const int4 v = __ldg(reinterpret_cast<const int4*>(p.rows) + col0 + row);
-      rd[i] = RowDesc{v.x, v.y, v.z, v.w};
+      rd[i] = row_at(p, rr, col0 + row);
     }
+    dep_wait(p);  // pool h/c and feed tokens are written by earlier launches
+    // device span starts when the launch's dependent work may begin (after the PDL wait)
+    if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
+    if (tid == 0 && p.tl != nullptr) atomicMax(p.tl + 1, ~gtimer());
+    if (tid == 0) phase_mark(p, 8);
 #pragma unroll
     for (int i = 0; i < kItems; ++i) {
       const int q = tid + i * kProducerThreads;
@@ -346,7 +398,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (tid == 0) phase_mark(p, 3);
     const int v0 = blockIdx.y * 128;
     for (int c = tid; c < ncols; c += kThreads) {
-      const RowDesc r = p.rows[col0 + c];
+      const RowDesc r = row_at(p, rr, col0 + c);
       float best = -INFINITY;
       int besti = 0;
       float* lg = nullptr;
@@ -378,15 +430,18 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (*flag_last) {  // last CTA: publish argmax -> feed token + emitted token, reset keys
       __threadfence();
       for (int c = tid; c < p.b; c += kThreads) {
-        const RowDesc r = p.rows[c];
+        const RowDesc r = row_at(p, rr, c);
         const unsigned long long key = atomicExch(p.amax + c, 0ull);
         const int y = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(key & 0xFFFFFFFFull));
         p.tok[r.slot] = y;
         p.res_tok[static_cast<size_t>(r.flags >> 8) * p.max_decode + r.b] = y;
       }
+      __threadfence();
       __syncthreads();
       if (tid == 0) {
         *p.done_ctas = 0;
+        __threadfence();
+        if (p.dep_flag != nullptr) st_release_gpu(p.dep_flag, p.dep_seq);
         if (p.signal != nullptr) {  // completion signal (A12) fused into the last CTA
           __threadfence_system();
           atomicAdd_system(p.signal, 1ull);
@@ -468,8 +523,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         if (p.experiment & 16) {  // diagnostics: no row / cell-state loads (garbage results)
           r = RowDesc{0, 0, (c_lo + cl) & 1023, 0};
         } else {
-          const int4 rv = __ldg(reinterpret_cast<const int4*>(p.rows) + col0 + c_lo + cl);
-          r = RowDesc{rv.x, rv.y, rv.z, rv.w};
+          r = row_at(p, rr, col0 + c_lo + cl);
         }
         const int u = unit0 + j;
         float hn, cn;
@@ -500,17 +554,10 @@ __global__ void __launch_bounds__(kThreads, 2)
     cluster_sync();  // B: peers may read this CTA's partials until here
     if (tid == 0) phase_mark(p, 5);
     if (tid == 0 && p.phase != nullptr) p.phase[(blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z)) * 64 + 15] = clock64();
-    if (p.signal != nullptr) {  // completion signal (A12) fused into the task's last CTA
+    if (p.dep_flag != nullptr || p.signal != nullptr) {
       __threadfence();
       __syncthreads();
-      if (tid == 0) {
-        const unsigned total = gridDim.x * gridDim.y * gridDim.z;
-        if (atomicAdd(p.sig_ctas, 1u) == total - 1) {
-          *p.sig_ctas = 0;
-          __threadfence_system();
-          atomicAdd_system(p.signal, 1ull);
-        }
-      }
+      launch_done(p, p.sig_ctas);
     }
   }
 
@@ -542,7 +589,7 @@ __global__ void __launch_bounds__(kThreads, 2)
 }
 
 template <int EPI>
-cudaError_t launch_impl(StepArgs a, cudaStream_t st) {
+cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   static bool configured = false;
   if (!configured) {
     cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI>,
@@ -575,18 +622,26 @@ cudaError_t launch_impl(StepArgs a, cudaStream_t st) {
   attr[1].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
-  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI>, a);
+  static thread_local StepRows inline_rows;
+  if (rows_host != nullptr) {
+    if (a.b > kMaxRowsInline) return cudaErrorInvalidValue;
+    memcpy(inline_rows.r, rows_host, sizeof(RowDesc) * a.b);
+    a.rows = nullptr;
+  } else if (a.rows == nullptr) {
+    return cudaErrorInvalidValue;
+  }
+  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI>, a, inline_rows);
 }
 
 }  // namespace
 
-cudaError_t launch_cell_step_sm100(const StepArgs& a, cudaStream_t st) {
+cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st) {
   if (a.b <= 0) return cudaSuccess;
   switch (a.epi) {
-    case EPI_LSTM: return launch_impl<EPI_LSTM>(a, st);
-    case EPI_LEAF: return launch_impl<EPI_LEAF>(a, st);
-    case EPI_INTERNAL: return launch_impl<EPI_INTERNAL>(a, st);
-    case EPI_PROJ: return launch_impl<EPI_PROJ>(a, st);
+    case EPI_LSTM: return launch_impl<EPI_LSTM>(a, rows_host, st);
+    case EPI_LEAF: return launch_impl<EPI_LEAF>(a, rows_host, st);
+    case EPI_INTERNAL: return launch_impl<EPI_INTERNAL>(a, rows_host, st);
+    case EPI_PROJ: return launch_impl<EPI_PROJ>(a, rows_host, st);
   }
   return cudaErrorInvalidValue;
 }

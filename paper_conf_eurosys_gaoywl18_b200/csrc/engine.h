@@ -188,7 +188,10 @@ struct Engine {
   int logits_vocab = 0;
   unsigned long long* amax = nullptr;
   unsigned int* done_ctas = nullptr;
-  unsigned int* sig_ctas = nullptr;  // CTA counter of the fused completion signal
+  unsigned int* sig_ctas = nullptr;  // CTA counter of the fused completion signal / chain flag
+  unsigned int* dep_flag = nullptr;  // launch chain flag (device): last completed sm100 launch
+  unsigned int dep_seq = 0;          // host: sequence number of the last sm100 launch issued
+  bool pdl_ok = false;               // the stream's last op was an sm100 launch (PDL is safe)
   RowDesc* ring_dev = nullptr;
   RowDesc* ring_host = nullptr;    // pinned staging
   int ring_rows = 0;

@@ -68,6 +68,8 @@ struct StepArgs {
                               // activation ring bytes
   unsigned long long* span;   // time_kernels: slot {min CTA start, CTAs done} (device memory)
   unsigned long long* span_acc;  // {sum of launch spans in ns, launches}: last CTA adds
+  unsigned int* dep_flag;     // launch chain: sequence number of the last completed launch
+  unsigned int dep_seq;       // this launch's sequence number (waits for dep_seq - 1)
   unsigned long long* tl;     // diagnostics (BM_TIMELINE): {~first CTA start, ~first past the
                               // PDL wait, last CTA end, CTAs} in %globaltimer ns, or null
 };
@@ -103,7 +105,16 @@ int persistent_smem_bytes();
 
 // bf16 / tcgen05 path (cell_step_sm100.cu). a.W: weights in the stage-tile layout
 // (launch_pack_tiles): [tile][K/64][tile_rows][64] bf16, 128B-swizzled rows.
-cudaError_t launch_cell_step_sm100(const StepArgs& a, cudaStream_t st);
+// Row descriptors of one launch passed by value as a kernel parameter (the launch carries them:
+// no host->device copy and no cross-stream dependency between consecutive launches, so PDL
+// overlaps a launch's prologue with the previous launch's tail).
+constexpr int kMaxRowsInline = 512;
+struct StepRows {
+  RowDesc r[kMaxRowsInline];
+};
+// rows_host: the launch's rows in host memory (b <= kMaxRowsInline) -- passed inline; or null,
+// then a.rows must point to device memory holding them.
+cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st);
 // fp32 / SIMT path (cell_step_simt.cu)
 cudaError_t launch_cell_step_simt(const StepArgs& a, cudaStream_t st);
 

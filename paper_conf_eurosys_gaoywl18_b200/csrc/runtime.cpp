@@ -69,8 +69,8 @@ void algo_cost(const Engine& e, const Cell& c, int b, bool proj, double* bytes, 
 }  // namespace
 
 // ---------------------------------------------------------------- launching tasks
-static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, int b, int layer,
-                                 bool proj, int* ev_out, unsigned long long* signal) {
+static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, const RowDesc* rows_host,
+                                 int b, int layer, bool proj, int* ev_out, unsigned long long* signal) {
   StepArgs a{};
   a.epi = proj ? EPI_PROJ : c.epi;
   a.G = proj ? 1 : c.G;
@@ -118,8 +118,15 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
   a.experiment = experiment;
   a.signal = signal;
   a.sig_ctas = e.sig_ctas;
+  // PDL only directly behind another tcgen05 launch: the chain flag orders launches among
+  // themselves, while copies / other kernels before a launch need full stream ordering
   static const int no_pdl = getenv("BM_NO_PDL") ? atoi(getenv("BM_NO_PDL")) : 0;
-  a.pdl = no_pdl ? 0 : 1;
+  static const int no_chain = getenv("BM_NO_CHAIN") ? atoi(getenv("BM_NO_CHAIN")) : 0;
+  a.pdl = (no_pdl || !e.pdl_ok) ? 0 : 1;
+  if (!no_chain) {
+    a.dep_flag = e.dep_flag;
+    a.dep_seq = e.dep_seq + 1;
+  }
   TimedLaunch* tl = nullptr;
   // events serialise the stream and so disable PDL overlap around the launches they bracket:
   // time a sample (every kTimeEvery-th launch) instead of every launch
@@ -144,7 +151,11 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
   }
   cudaError_t err;
   if (e.cfg.precision == BM_PREC_BF16) {
-    err = launch_cell_step_sm100(a, e.stream);
+    err = launch_cell_step_sm100(a, rows_host, e.stream);
+    if (err == cudaSuccess) {
+      if (!no_chain) e.dep_seq += 1;
+      e.pdl_ok = true;
+    }
   } else {
     a.pdl = 0;  // the SIMT kernels do not use griddepcontrol
     err = launch_cell_step_simt(a, e.stream);
@@ -158,8 +169,8 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, in
 // All kernels of one task in order on the engine stream (§5). With `signal`, the task's
 // completion is signalled: fused into the last kernel's last CTA on the tcgen05 path (A12),
 // or by the signal kernel on the fp32 path.
-static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, int b, Task* t,
-                             unsigned long long* signal) {
+static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const RowDesc* rows_host, int b,
+                             Task* t, unsigned long long* signal) {
   const bool lstm = c.epi == EPI_LSTM;
   const bool proj = c.d.kind == BM_CELL_LSTM_PROJ;
   const bool fused = e.cfg.precision == BM_PREC_BF16;
@@ -167,7 +178,7 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, int b,
   for (int l = 0; l < L; ++l) {
     int ev = -1;
     const bool last = l == L - 1 && !proj;
-    bm_status s = launch_one_step(e, c, rows_dev, b, l, false, &ev, (last && fused) ? signal : nullptr);
+    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, l, false, &ev, (last && fused) ? signal : nullptr);
     if (s != BM_OK) return s;
     if (t && ev >= 0) {
       if (t->ev_first < 0) t->ev_first = ev;
@@ -176,7 +187,7 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, int b,
   }
   if (proj) {
     int ev = -1;
-    bm_status s = launch_one_step(e, c, rows_dev, b, 0, true, &ev, fused ? signal : nullptr);
+    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, 0, true, &ev, fused ? signal : nullptr);
     if (s != BM_OK) return s;
     if (t && ev >= 0) t->ev_count += 1;
   }
@@ -213,6 +224,14 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
     }
   }
   if (!e.device()) return BM_OK;
+  if (e.cfg.precision == BM_PREC_BF16 && !e.persistent_active) {
+    // tcgen05 path: each launch carries its task's row descriptors as a kernel parameter
+    for (Task& t : tasks) {
+      bm_status s = launch_cell(e, e.cells[t.ct], nullptr, t.desc.data(), t.b, &t, e.signal_dev);
+      if (s != BM_OK) return s;
+    }
+    return BM_OK;
+  }
   // ring placement: one contiguous region for all tasks of this Schedule call
   if (total > e.ring_rows) return BM_E_INVAL;
   if (e.ring_head + total > e.ring_rows) e.ring_head = 0;
@@ -261,7 +280,7 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
   CK(cudaEventRecord(e.copy_ev, e.copy_stream));
   CK(cudaStreamWaitEvent(e.stream, e.copy_ev, 0));
   for (Task& t : tasks) {
-    bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, t.b, &t, e.signal_dev);
+    bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, nullptr, t.b, &t, e.signal_dev);
     if (s != BM_OK) return s;
   }
   return BM_OK;
@@ -430,6 +449,7 @@ static void free_device(Engine& e) {
   cudaFree(e.amax);
   cudaFree(e.done_ctas);
   cudaFree(e.sig_ctas);
+  cudaFree(e.dep_flag);
   cudaFree(e.ring_dev);
   cudaFree(e.direct_rows);
   cudaFree(e.phase_dev);
@@ -491,7 +511,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
               dalloc(&E.res_h, R * L * H) == cudaSuccess && dalloc(&E.res_c, R * L * H) == cudaSuccess &&
               dalloc(&E.res_tok, R * static_cast<size_t>(c.max_decode_len)) == cudaSuccess &&
               dalloc(&E.amax, 512) == cudaSuccess && dalloc(&E.done_ctas, 1) == cudaSuccess &&
-              dalloc(&E.sig_ctas, 1) == cudaSuccess &&
+              dalloc(&E.sig_ctas, 1) == cudaSuccess && dalloc(&E.dep_flag, 1) == cudaSuccess &&
               dalloc(&E.direct_rows, 2 * 4096) == cudaSuccess &&
               cudaEventCreateWithFlags(&E.direct_ev[0], cudaEventDisableTiming) == cudaSuccess &&
               cudaEventCreateWithFlags(&E.direct_ev[1], cudaEventDisableTiming) == cudaSuccess;
@@ -513,6 +533,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
         cudaMemsetAsync(E.amax, 0, 512 * 8, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.done_ctas, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.sig_ctas, 0, 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.dep_flag, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.res_tok, 0, R * c.max_decode_len * 4, E.stream) != cudaSuccess)
       return fail(BM_E_CUDA);
     if (c.time_kernels) {
@@ -556,6 +577,7 @@ void* bm_stream(bm_engine* h) { return h ? reinterpret_cast<Engine*>(h)->stream 
 bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w, int* cell_id) {
   if (h == nullptr || d == nullptr || w == nullptr || cell_id == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (e.sticky_cuda) return BM_E_CUDA;
   if (e.submitted_any) return BM_E_STATE;
   if (e.cells.size() >= 64) return BM_E_INVAL;
@@ -789,6 +811,7 @@ static bool persistent_eligible(const Engine& e) {
 }
 
 static bm_status persistent_start(Engine& e) {
+  e.pdl_ok = false;
   const Cell& c = e.cells[0];
   if (e.hdr_dev == nullptr) {
     CK(cudaMalloc(&e.hdr_dev, sizeof(TaskHdr) * e.hdr_ring));
@@ -841,6 +864,7 @@ static bm_status persistent_start(Engine& e) {
 }
 
 static bm_status persistent_stop(Engine& e) {
+  e.pdl_ok = false;
   if (!e.persistent_active) return BM_OK;
   const int idx = static_cast<int>((e.launched - e.run_base) % e.hdr_ring);
   // the slot's previous task retired long ago (at most k + MaxTasksToSubmit are in flight)
@@ -924,6 +948,7 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
 bm_status bm_read_result(bm_engine* h, uint64_t req_id, bm_result* dst) {
   if (h == nullptr || dst == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (e.sticky_cuda) return BM_E_CUDA;
   Request& r = e.reqs[req_id % e.cfg.max_requests];
   if (!r.used || r.id != req_id) return BM_E_INVAL;
@@ -962,6 +987,7 @@ bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh
                                int release) {
   if (h == nullptr || n < 1) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (e.sticky_cuda) return BM_E_CUDA;
   if (!e.device()) return BM_E_STATE;
   const uint64_t R = e.cfg.max_requests;
@@ -1022,27 +1048,38 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
     if (rows[i].slot < 0 || rows[i].slot >= e.cfg.max_slots) return BM_E_INVAL;
     if ((rows[i].flags >> 8) >= e.cfg.max_requests) return BM_E_INVAL;
   }
-  // stage through pinned memory so the copy is truly asynchronous (back-to-back direct steps)
+  // tcgen05 path, b <= 512: the rows travel inline with the launch
+  const bool inline_rows = e.cfg.precision == BM_PREC_BF16 && b <= kMaxRowsInline;
+  const RowDesc* rows_host = inline_rows ? reinterpret_cast<const RowDesc*>(rows) : nullptr;
+  // otherwise stage through pinned memory so the copy is truly asynchronous (back-to-back steps)
   if (e.direct_host == nullptr)
     CK(cudaHostAlloc(reinterpret_cast<void**>(&e.direct_host), sizeof(RowDesc) * 4096 * 2, cudaHostAllocDefault));
-  RowDesc* stage = e.direct_host + (e.direct_flip ^= 1) * 4096;
-  if (async) CK(cudaEventSynchronize(e.direct_ev[e.direct_flip]));
-  memcpy(stage, rows, sizeof(RowDesc) * b);
-  CK(cudaMemcpyAsync(e.direct_rows + e.direct_flip * 4096, stage, sizeof(RowDesc) * b, cudaMemcpyHostToDevice, e.stream));
-  CK(cudaEventRecord(e.direct_ev[e.direct_flip], e.stream));
-  RowDesc* rows_dev = e.direct_rows + e.direct_flip * 4096;
+  RowDesc* rows_dev = nullptr;
+  if (!inline_rows) {
+    e.pdl_ok = false;
+    RowDesc* stage = e.direct_host + (e.direct_flip ^= 1) * 4096;
+    if (async) CK(cudaEventSynchronize(e.direct_ev[e.direct_flip]));
+    memcpy(stage, rows, sizeof(RowDesc) * b);
+    CK(cudaMemcpyAsync(e.direct_rows + e.direct_flip * 4096, stage, sizeof(RowDesc) * b, cudaMemcpyHostToDevice,
+                       e.stream));
+    CK(cudaEventRecord(e.direct_ev[e.direct_flip], e.stream));
+    rows_dev = e.direct_rows + e.direct_flip * 4096;
+  }
   // diagnostics: BM_REPEAT=n launches the step n times back to back (steady-state throughput
   // with PDL overlap between consecutive launches; the state advances n steps)
   static const int repeat = getenv("BM_REPEAT") ? atoi(getenv("BM_REPEAT")) : 1;
   for (int rep = 1; rep < repeat; ++rep) {
-    bm_status s0 = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
+    bm_status s0 = launch_cell(e, c, rows_dev, rows_host, b, nullptr, nullptr);
     if (s0 != BM_OK) return s0;
   }
   // diagnostics: BM_PHASE_DUMP=<file> records per-CTA phase timestamps of every direct step
   static const char* dump = getenv("BM_PHASE_DUMP");
   if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 64 * 4096));
-  if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 64 * 4096, e.stream));
-  bm_status s = launch_cell(e, c, rows_dev, b, nullptr, nullptr);
+  if (e.phase_dev) {
+    CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 64 * 4096, e.stream));
+    e.pdl_ok = false;
+  }
+  bm_status s = launch_cell(e, c, rows_dev, rows_host, b, nullptr, nullptr);
   if (s != BM_OK) return s;
   if (!async || e.phase_dev) CK(cudaStreamSynchronize(e.stream));
   if (e.phase_dev) {
@@ -1065,6 +1102,7 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
 
 static bm_status pool_io(Engine& e, int layer, int parity, const int32_t* slots, int n, float* h,
                          float* c, int write) {
+  e.pdl_ok = false;
   if (!e.device()) return BM_E_STATE;
   if (layer < 0 || layer >= e.cfg.pool_layers || parity < 0 || parity > 1 || n < 1 || slots == nullptr)
     return BM_E_INVAL;
@@ -1114,6 +1152,7 @@ bm_status bm_pool_read(bm_engine* h, int layer, int parity, const int32_t* slots
 bm_status bm_result_rows(bm_engine* h, const int32_t* res_idx, int n, float* hh, float* cc) {
   if (h == nullptr || res_idx == nullptr || n < 1) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (!e.device()) return BM_E_STATE;
   const size_t LH = e.H() * e.cfg.pool_layers;
   CK(cudaStreamSynchronize(e.stream));
@@ -1129,6 +1168,7 @@ bm_status bm_result_rows(bm_engine* h, const int32_t* res_idx, int n, float* hh,
 bm_status bm_tokens(bm_engine* h, const int32_t* slots, int n, int32_t* inout, int write) {
   if (h == nullptr || slots == nullptr || inout == nullptr || n < 1) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (!e.device()) return BM_E_STATE;
   CK(cudaStreamSynchronize(e.stream));
   for (int i = 0; i < n; ++i) {
