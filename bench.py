@@ -77,7 +77,7 @@ def parse():
 WL = {
     "lstm": dict(config="BASELINE configs[1]: 1-layer LSTM h=1024, WMT-like lengths, Poisson arrivals, "
                         "bmax 512, 1 B200", hidden=1024, layers=1, vocab=32768, reqs=20000,
-                 p90_ms=12.0, lookahead=2, persistent=1),
+                 p90_ms=12.0, lookahead=2, persistent=0),
     "seq2seq": dict(config="BASELINE configs[2]: Seq2Seq 4+4 layer LSTM h=1024, vocab 32768, greedy "
                            "decode, encoder/decoder bmax 512/256", hidden=1024, layers=4, vocab=32768,
                     reqs=4000, p90_ms=None, lookahead=1, persistent=0),

@@ -37,7 +37,7 @@ namespace {
 using namespace ptx;
 
 constexpr int kMaxStages = 8;           // pipeline depth cap
-constexpr int kTailBytes = 1024;        // barriers + TMEM slot, at smem offset 0
+constexpr int kTailBytes = 5120;        // barriers + TMEM slot (1 KB), row table [256] (4 KB)
 constexpr int kBK = 64;                 // K elements per stage (128 B of bf16 = one SW128 atom)
 constexpr int kProducerThreads = 256;   // warps 0-7: activation gather (cp.async)
 constexpr int kMmaWarp = 8;             // warp 8: TMEM alloc + tcgen05.mma issue
@@ -62,7 +62,7 @@ constexpr int kWRing = 2;               // weight chunks in the ring
 // in ~100 KB and two CTAs share an SM: under PDL the next launch's weight stream and gather
 // overlap this launch's split-K epilogue. Larger tasks use 64 KB chunks and a 64 KB ring.
 // Default plan; the launcher passes the chosen chunk size / ring size in StepArgs.
-__host__ __device__ __forceinline__ int w_chunk_blocks(int npad) { return npad <= 128 ? 2 : kWChunkMax; }
+__host__ __device__ __forceinline__ int w_chunk_blocks(int) { return kWChunkMax; }
 __host__ __device__ __forceinline__ int x_ring_bytes(int npad) { return npad <= 128 ? 32 * 1024 : 64 * 1024; }
 __host__ __device__ __forceinline__ int x_stages_for(int npad, int xring) {
   const int n = xring / (npad * 128);
@@ -208,7 +208,8 @@ __global__ void __launch_bounds__(kThreads, 2)
   const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages + 2 * kWRing);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 2 * kWRing + 1);
   int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
-  uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 1 KB)
+  RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);  // this CTA's rows (col0 + c)
+  uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
   uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
   uint8_t* x_st = smem + kWRing * wcb * kWStageBytes;     // kStages x npad x 128 B
   const int x_stage_bytes = npad * 128;
@@ -255,10 +256,15 @@ __global__ void __launch_bounds__(kThreads, 2)
     const __nv_bfloat16* src1[kItems];
     uint32_t dst_off[kItems];
     RowDesc rd[kItems];
+    // the launch's own rows (independent of earlier launches) into the smem table: one 16-byte
+    // parameter load per thread (parameter loads miss the constant cache and serialise per
+    // address: each row is read once and then shared through shared memory)
+    if (tid < ncols) rtab[tid] = row_at(p, rr, col0 + tid);
+    named_bar(1, kProducerThreads);
 #pragma unroll
-    for (int i = 0; i < kItems; ++i) {  // the launch's own rows: independent of earlier launches
+    for (int i = 0; i < kItems; ++i) {
       const int row = min((tid + i * kProducerThreads) >> 3, ncols - 1);
-      rd[i] = row_at(p, rr, col0 + row);
+      rd[i] = rtab[row];
     }
     dep_wait(p);  // pool h/c and feed tokens are written by earlier launches
     // device span starts when the launch's dependent work may begin (after the PDL wait)
@@ -398,7 +404,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (tid == 0) phase_mark(p, 3);
     const int v0 = blockIdx.y * 128;
     for (int c = tid; c < ncols; c += kThreads) {
-      const RowDesc r = row_at(p, rr, col0 + c);
+      const RowDesc r = rtab[c];
       float best = -INFINITY;
       int besti = 0;
       float* lg = nullptr;
@@ -523,7 +529,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         if (p.experiment & 16) {  // diagnostics: no row / cell-state loads (garbage results)
           r = RowDesc{0, 0, (c_lo + cl) & 1023, 0};
         } else {
-          r = row_at(p, rr, col0 + c_lo + cl);
+          r = rtab[c_lo + cl];
         }
         const int u = unit0 + j;
         float hn, cn;
