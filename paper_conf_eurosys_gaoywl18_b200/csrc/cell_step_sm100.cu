@@ -69,13 +69,18 @@ __host__ __device__ __forceinline__ int x_stages_for(int npad, int xring) {
   return n < 2 ? 2 : (n > kMaxStages ? kMaxStages : n);
 }
 // weight ring + activation ring, reused after the main loop for the partial / logits tile
-__host__ __device__ __forceinline__ int region_bytes(int npad, int wcb, int xring) {
-  const int a = kWRing * wcb * kWStageBytes + x_stages_for(npad, xring) * npad * 128;
+// wblk = one K block of the CTA's weight tile (tile rows x 128 B: 16 KB LSTM / projection,
+// 12 KB leaf, 10 KB internal)
+__host__ __device__ __forceinline__ int region_bytes(int npad, int wcb, int xring, int wblk) {
+  const int a = kWRing * wcb * wblk + x_stages_for(npad, xring) * npad * 128;
   const int b = 129 * npad * 4 + 4 * 128 * 4;
   return a > b ? a : b;
 }
 
-__device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
+// Gate nonlinearities: ex2/rcp approximations (MUFU), absolute error ~1e-7 -- far inside the
+// bf16 path's 5e-3 bound -- without the IEEE-division / tanhf slow paths.
+__device__ __forceinline__ float sigm(float x) { return __fdividef(1.0f, 1.0f + __expf(-x)); }
+__device__ __forceinline__ float tanh_f(float x) { return 1.0f - __fdividef(2.0f, __expf(2.0f * x) + 1.0f); }
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -211,7 +216,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);  // this CTA's rows (col0 + c)
   uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
   uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
-  uint8_t* x_st = smem + kWRing * wcb * kWStageBytes;     // kStages x npad x 128 B
+  uint8_t* x_st = smem + kWRing * wcb * wblk_bytes;       // kStages x npad x 128 B
   const int x_stage_bytes = npad * 128;
 
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
@@ -340,7 +345,7 @@ __global__ void __launch_bounds__(kThreads, 2)
                      : "memory");
         // one chunk = nblk consecutive K blocks (contiguous in the stage-tile layout); block i
         // lands at i * wblk_bytes (a multiple of 1024: the 128B-swizzle atom stays aligned)
-        bulk_load(smem_u32(w_ring + s * wcb * kWStageBytes),
+        bulk_load(smem_u32(w_ring + s * wcb * wblk_bytes),
                   wsrc + static_cast<size_t>(c) * kpc * wblk_bytes, bytes, wfull0 + 8 * s);
       }
     }
@@ -363,7 +368,7 @@ __global__ void __launch_bounds__(kThreads, 2)
       if (lane == 0 && kb % kpc == 0 && c < 4) phase_mark(p, 28 + c);  // weight chunk c at the MMA
       if (lane == 0) {
         const uint64_t a =
-            sdesc_sw128(smem_u32(w_ring + ws * wcb * kWStageBytes + (kb % kpc) * wblk_bytes));
+            sdesc_sw128(smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
         const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes));
         if (!(p.experiment & 8)) {  // diagnostics bit 8: no MMA instructions
 #pragma unroll
@@ -494,65 +499,90 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int prow0 = blockIdx.y * tile_rows;
     const size_t H = p.H;
     const size_t NS = p.n_slots;
-    if (warp < 8) {
-      const int cols_per_pass = kProducerThreads / U;
+    {
+      // every warp takes part; each thread owns unit j of columns cl0, cl0 + step, ... and
+      // handles two columns per iteration with all their loads issued up front (ILP: the
+      // DSMEM round trip, not the arithmetic, bounds an iteration)
+      const int ew = kThreads / U;  // columns per pass (LSTM/leaf U = 32: 10, internal U = 16: 20)
       const int j = tid % U;
+      const int u = unit0 + j;
       float bias[5];
 #pragma unroll
       for (int g = 0; g < 5; ++g) bias[g] = g < G ? p.bias[prow0 + j * G + g] : 0.f;
-      for (int cl = tid / U; cl < my_cols; cl += cols_per_pass) {
-        if (tid == 0 && cl / cols_per_pass < 16) phase_mark(p, 32 + cl / cols_per_pass);
-        float z[5];
+      const bool no_dsmem = (p.experiment & 32) != 0;  // diagnostics: own partial only
+      for (int cl = tid / U; cl < my_cols; cl += 2 * ew) {
+        if (tid == 0 && cl / (2 * ew) < 16) phase_mark(p, 32 + cl / (2 * ew));
+        const int nit = (cl + ew < my_cols) ? 2 : 1;
+        float4 v[2][kMaxS], w[2][kMaxS];
+        RowDesc r[2];
+        float cin[2][2];
 #pragma unroll
-        for (int g = 0; g < 5; ++g) z[g] = bias[g];
-        const uint32_t off = static_cast<uint32_t>(((c_lo + cl) * pitch + j * Gp) * 4);
-        // issue every remote load of this item before using any, then add in fixed order
-        float4 v[kMaxS], w[kMaxS];
-        const bool no_dsmem = (p.experiment & 32) != 0;  // diagnostics: own partial only
+        for (int h = 0; h < 2; ++h) {
+          if (h < nit) {
+            const uint32_t off = static_cast<uint32_t>(((c_lo + cl + h * ew) * pitch + j * Gp) * 4);
 #pragma unroll
-        for (int s = 0; s < kMaxS; ++s)
-          if (s < S) {
-            const uint32_t a = no_dsmem ? smem_u32(P) + off : peer[s] + off;
-            v[s] = ld_cluster_v4(a);
-            if (G == 5) w[s] = ld_cluster_v4(a + 16);
+            for (int s = 0; s < kMaxS; ++s)
+              if (s < S) {
+                const uint32_t a = no_dsmem ? smem_u32(P) + off : peer[s] + off;
+                v[h][s] = ld_cluster_v4(a);
+                if (G == 5) w[h][s] = ld_cluster_v4(a + 16);
+              }
+            r[h] = (p.experiment & 16) ? RowDesc{0, 0, (c_lo + cl + h * ew) & 1023, 0} : rtab[c_lo + cl + h * ew];
+            cin[h][0] = cin[h][1] = 0.f;
+            if (!(p.experiment & 16)) {
+              if constexpr (EPI == EPI_LSTM) {
+                if (!(r[h].flags & ROW_FIRST)) cin[h][0] = p.c_pool[r[h].slot * H + u];
+              } else if constexpr (EPI == EPI_INTERNAL) {
+                cin[h][0] = p.c_pool[static_cast<size_t>(r[h].a) * H + u];
+                cin[h][1] = p.c_pool[static_cast<size_t>(r[h].b) * H + u];
+              }
+            }
           }
+        }
 #pragma unroll
-        for (int s = 0; s < kMaxS; ++s)
-          if (s < S) {
-            z[0] += v[s].x;
-            z[1] += v[s].y;
-            z[2] += v[s].z;
-            if (G >= 4) z[3] += v[s].w;
-            if (G == 5) z[4] += w[s].x;
+        for (int h = 0; h < 2; ++h) {
+          if (h < nit) {
+            float z[5];
+#pragma unroll
+            for (int g = 0; g < 5; ++g) z[g] = bias[g];
+#pragma unroll
+            for (int s = 0; s < kMaxS; ++s)  // fixed order s = 0..S-1 (batch invariance)
+              if (s < S) {
+                z[0] += v[h][s].x;
+                z[1] += v[h][s].y;
+                z[2] += v[h][s].z;
+                if (G >= 4) z[3] += v[h][s].w;
+                if (G == 5) z[4] += w[h][s].x;
+              }
+            float hn, cn;
+            if constexpr (EPI == EPI_LSTM) {
+              cn = sigm(z[1]) * cin[h][0] + sigm(z[0]) * tanh_f(z[2]);
+              hn = sigm(z[3]) * tanh_f(cn);
+            } else if constexpr (EPI == EPI_LEAF) {
+              cn = sigm(z[0]) * tanh_f(z[2]);
+              hn = sigm(z[1]) * tanh_f(cn);
+            } else {
+              cn = sigm(z[0]) * tanh_f(z[4]) + sigm(z[1]) * cin[h][0] + sigm(z[2]) * cin[h][1];
+              hn = sigm(z[3]) * tanh_f(cn);
+            }
+            if (p.experiment & 256) {  // diagnostics: no gate math
+              cn = z[0] + z[1];
+              hn = z[2] + z[3];
+            }
+            if (p.experiment & 128) {  // diagnostics: no stores (keep the values live)
+              if (cn == 12345.f && hn == 54321.f) p.c_pool[0] = cn;
+              continue;
+            }
+            const RowDesc& rr_ = r[h];
+            p.c_pool[rr_.slot * H + u] = cn;
+            const int par_out = (EPI == EPI_LSTM) ? ((rr_.flags & ROW_PARITY) ? 0 : 1) : 0;
+            static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + rr_.slot) * H + u] = __float2bfloat16_rn(hn);
+            if (rr_.flags & ROW_LAST) {
+              const size_t ro = (static_cast<size_t>(rr_.flags >> 8) * p.res_layers + p.layer) * H + u;
+              p.res_h[ro] = hn;
+              p.res_c[ro] = cn;
+            }
           }
-        RowDesc r;
-        if (p.experiment & 16) {  // diagnostics: no row / cell-state loads (garbage results)
-          r = RowDesc{0, 0, (c_lo + cl) & 1023, 0};
-        } else {
-          r = rtab[c_lo + cl];
-        }
-        const int u = unit0 + j;
-        float hn, cn;
-        if constexpr (EPI == EPI_LSTM) {
-          const float cp = ((r.flags & ROW_FIRST) || (p.experiment & 16)) ? 0.f : p.c_pool[r.slot * H + u];
-          cn = sigm(z[1]) * cp + sigm(z[0]) * tanhf(z[2]);
-          hn = sigm(z[3]) * tanhf(cn);
-        } else if constexpr (EPI == EPI_LEAF) {
-          cn = sigm(z[0]) * tanhf(z[2]);
-          hn = sigm(z[1]) * tanhf(cn);
-        } else {
-          const float cl_ = (p.experiment & 16) ? 0.f : p.c_pool[static_cast<size_t>(r.a) * H + u];
-          const float cr_ = (p.experiment & 16) ? 0.f : p.c_pool[static_cast<size_t>(r.b) * H + u];
-          cn = sigm(z[0]) * tanhf(z[4]) + sigm(z[1]) * cl_ + sigm(z[2]) * cr_;
-          hn = sigm(z[3]) * tanhf(cn);
-        }
-        p.c_pool[r.slot * H + u] = cn;
-        const int par_out = (EPI == EPI_LSTM) ? ((r.flags & ROW_PARITY) ? 0 : 1) : 0;
-        static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + r.slot) * H + u] = __float2bfloat16_rn(hn);
-        if (r.flags & ROW_LAST) {
-          const size_t ro = (static_cast<size_t>(r.flags >> 8) * p.res_layers + p.layer) * H + u;
-          p.res_h[ro] = hn;
-          p.res_c[ro] = cn;
         }
       }
     }
@@ -608,9 +638,13 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   // ring plan (BM_WCB = K blocks per weight chunk, BM_XRING = activation ring KB: experiments)
   static const int env_wcb = getenv("BM_WCB") ? atoi(getenv("BM_WCB")) : 0;
   static const int env_xring = getenv("BM_XRING") ? atoi(getenv("BM_XRING")) : 0;
-  a.wcb = env_wcb > 0 ? env_wcb : w_chunk_blocks(npad);
-  a.xring = env_xring > 0 ? env_xring * 1024 : x_ring_bytes(npad);
-  const size_t smem = 1024 + kTailBytes + region_bytes(npad, a.wcb, a.xring);
+  // internal cells launch 64 tiles x 4 = 256 CTAs: their plan keeps two CTAs per SM (one
+  // wave) -- the whole 80 KB slice + a 24 KB activation ring up to 64 rows, half the slice above
+  const bool internal = EPI == EPI_INTERNAL;
+  a.wcb = env_wcb > 0 ? env_wcb : (internal && npad > 64 ? 2 : w_chunk_blocks(npad));
+  a.xring = env_xring > 0 ? env_xring * 1024 : (internal && npad <= 64 ? 24 * 1024 : x_ring_bytes(npad));
+  const int wblk = (EPI == EPI_PROJ ? 128 : gates_of(EPI) * a.U) * 128;
+  const size_t smem = 1024 + kTailBytes + region_bytes(npad, a.wcb, a.xring, wblk);
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int S = EPI == EPI_PROJ ? 1 : a.S;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;
