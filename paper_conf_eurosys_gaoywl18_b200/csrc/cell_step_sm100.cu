@@ -71,8 +71,9 @@ __host__ __device__ __forceinline__ int x_stages_for(int npad, int xring) {
 // weight ring + activation ring, reused after the main loop for the partial / logits tile
 // wblk = one K block of the CTA's weight tile (tile rows x 128 B: 16 KB LSTM / projection,
 // 12 KB leaf, 10 KB internal)
-__host__ __device__ __forceinline__ int region_bytes(int npad, int wcb, int xring, int wblk) {
-  const int a = kWRing * wcb * wblk + x_stages_for(npad, xring) * npad * 128;
+// xkb = K blocks per activation stage (one hand-off per stage)
+__host__ __device__ __forceinline__ int region_bytes(int npad, int wcb, int xring, int wblk, int xkb) {
+  const int a = kWRing * wcb * wblk + x_stages_for(npad * xkb, xring) * npad * xkb * 128;
   const int b = 129 * npad * 4 + 4 * 128 * 4;
   return a > b ? a : b;
 }
@@ -197,8 +198,12 @@ __global__ void __launch_bounds__(kThreads, 2)
   const int npad = (ncols + 15) & ~15;
   const int nk = p.kslice / kBK;
   const int k_begin = static_cast<int>(rank) * p.kslice;
-  const int kStages = p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad, p.xring))
-                                       : x_stages_for(npad, p.xring);
+  // activation stages: xkb consecutive K blocks each, ONE producer -> MMA hand-off per stage
+  // (every mbarrier hand-off costs ~0.15-0.3 us of latency on the MMA's path, tools/pipe_bench.cu)
+  const int xkb = p.xkb > 0 ? p.xkb : 1;
+  const int nst = nk / xkb;
+  const int kStages = p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad * xkb, p.xring))
+                                       : x_stages_for(npad * xkb, p.xring);
   const int wcb = p.wcb;                                  // ring slot capacity in K blocks
   const int kpc = min(wcb, nk);                           // K blocks per weight chunk
   const int n_chunks = (nk + kpc - 1) / kpc;
@@ -216,8 +221,9 @@ __global__ void __launch_bounds__(kThreads, 2)
   RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);  // this CTA's rows (col0 + c)
   uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
   uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
-  uint8_t* x_st = smem + kWRing * wcb * wblk_bytes;       // kStages x npad x 128 B
-  const int x_stage_bytes = npad * 128;
+  uint8_t* x_st = smem + kWRing * wcb * wblk_bytes;       // kStages x xkb x npad x 128 B
+  const int x_blk_bytes = npad * 128;                     // one K block of the activation tile
+  const int x_stage_bytes = x_blk_bytes * xkb;
 
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
@@ -297,31 +303,33 @@ __global__ void __launch_bounds__(kThreads, 2)
     // (full barrier count = 256), so no producer waits on its own copies.
     const __nv_bfloat16* dummy = static_cast<const __nv_bfloat16*>(p.E != nullptr ? p.E : p.h_pool);
     const bool no_reads = (p.experiment & 1) != 0;
-    for (int kb = 0; kb < nk; ++kb) {
-      const int s = kb % kStages;
-      const int round = kb / kStages;
+    for (int st = 0; st < nst; ++st) {
+      const int s = st % kStages;
+      const int round = st / kStages;
       if (round > 0) mbar_wait_warp(empty0 + 8 * s, (round - 1) & 1);
-      const int k = k_begin + kb * kBK;
-      const int seg = k >= p.K0 ? 1 : 0;
-      const int kk = k - seg * p.K0;
-      const uint32_t xs = smem_u32(x_st + s * x_stage_bytes);
       if (p.experiment & 4) {  // diagnostics: no gather at all, hand the stage over at once
         mbar_arrive(full0 + 8 * s);
         continue;
       }
+      for (int j = 0; j < xkb; ++j) {
+        const int k = k_begin + (st * xkb + j) * kBK;
+        const int seg = k >= p.K0 ? 1 : 0;
+        const int kk = k - seg * p.K0;
+        const uint32_t xs = smem_u32(x_st + s * x_stage_bytes + j * x_blk_bytes);
 #pragma unroll
-      for (int i = 0; i < kItems; ++i) {
-        if (i < n_items) {
-          const __nv_bfloat16* src = seg ? src1[i] : src0[i];
-          if (src != nullptr && !no_reads) {
-            cp_async_16(xs + dst_off[i], src + kk, 16);
-          } else {
-            cp_async_16(xs + dst_off[i], dummy, 0);  // zero fill
+        for (int i = 0; i < kItems; ++i) {
+          if (i < n_items) {
+            const __nv_bfloat16* src = seg ? src1[i] : src0[i];
+            if (src != nullptr && !no_reads) {
+              cp_async_16(xs + dst_off[i], src + kk, 16);
+            } else {
+              cp_async_16(xs + dst_off[i], dummy, 0);  // zero fill
+            }
           }
         }
       }
       cp_async_arrive_noinc(full0 + 8 * s);
-      if (tid == 0 && kb == 0) phase_mark(p, 10);
+      if (tid == 0 && st == 0) phase_mark(p, 10);
     }
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
@@ -353,32 +361,41 @@ __global__ void __launch_bounds__(kThreads, 2)
   } else {
     // ================================================================ MMA issuer (A8)
     const uint32_t idesc = idesc_bf16(128, npad);
-    for (int kb = 0; kb < nk; ++kb) {
-      const int s = kb % kStages;
-      const int c = kb / kpc;
-      const int ws = c % kWRing;
-      if (kb % kpc == 0) mbar_wait_warp(wfull0 + 8 * ws, (c / kWRing) & 1);
-      if (lane == 0 && kb == 0) phase_mark(p, 13);
-      mbar_wait_warp(full0 + 8 * s, (kb / kStages) & 1);
+    for (int st = 0; st < nst; ++st) {
+      const int s = st % kStages;
+      mbar_wait_warp(full0 + 8 * s, (st / kStages) & 1);
       tc_fence_after();
-      if (lane == 0 && kb == 0) phase_mark(p, 6);
-      if (lane == 0 && kb == nk - 1) phase_mark(p, 7);
-      if (lane == 0 && kb == 1) phase_mark(p, 12);
-      if (lane == 0 && kb < 12) phase_mark(p, 16 + kb);   // stage kb at the MMA
-      if (lane == 0 && kb % kpc == 0 && c < 4) phase_mark(p, 28 + c);  // weight chunk c at the MMA
-      if (lane == 0) {
-        const uint64_t a =
-            sdesc_sw128(smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
-        const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes));
-        if (!(p.experiment & 8)) {  // diagnostics bit 8: no MMA instructions
-#pragma unroll
-          for (int k = 0; k < kBK / 16; ++k) {
-            mma_bf16(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
-          }
+      if (lane == 0 && st < 12) phase_mark(p, 16 + st);   // stage st at the MMA
+      if (lane == 0 && st == 0) phase_mark(p, 6);
+      if (lane == 0 && st == nst - 1) phase_mark(p, 7);
+      if (lane == 0 && st == 1) phase_mark(p, 12);
+      for (int j = 0; j < xkb; ++j) {
+        const int kb = st * xkb + j;
+        const int c = kb / kpc;
+        const int ws = c % kWRing;
+        if (kb % kpc == 0) {
+          mbar_wait_warp(wfull0 + 8 * ws, (c / kWRing) & 1);
+          tc_fence_after();
+          if (lane == 0 && c < 4) phase_mark(p, 28 + c);  // weight chunk c at the MMA
+          if (lane == 0 && kb == 0) phase_mark(p, 13);
         }
+        if (lane == 0) {
+          const uint64_t a =
+              sdesc_sw128(smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
+          const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes + j * x_blk_bytes));
+          if (!(p.experiment & 8)) {  // diagnostics bit 8: no MMA instructions
+#pragma unroll
+            for (int k = 0; k < kBK / 16; ++k) {
+              mma_bf16(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
+            }
+          }
+          if (kb % kpc == kpc - 1 || kb == nk - 1) mma_commit(wempty0 + 8 * ws);
+        }
+        __syncwarp();
+      }
+      if (lane == 0) {
         mma_commit(empty0 + 8 * s);
-        if (kb % kpc == kpc - 1 || kb == nk - 1) mma_commit(wempty0 + 8 * ws);
-        if (kb == nk - 1) mma_commit(done_bar);
+        if (st == nst - 1) mma_commit(done_bar);
       }
       __syncwarp();
     }
@@ -643,8 +660,23 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   const bool internal = EPI == EPI_INTERNAL;
   a.wcb = env_wcb > 0 ? env_wcb : (internal && npad > 64 ? 2 : w_chunk_blocks(npad));
   a.xring = env_xring > 0 ? env_xring * 1024 : (internal && npad <= 64 ? 24 * 1024 : x_ring_bytes(npad));
+  // K blocks per activation stage: fewer, larger hand-offs where shared memory allows (the
+  // 128-row LSTM / projection tiles keep a 128 KB weight slice + a 64 KB activation ring)
+  static const int env_xkb = getenv("BM_XKB") ? atoi(getenv("BM_XKB")) : 0;
+  a.xkb = 1;
+  if (!internal && EPI != EPI_LEAF) {
+    if (npad <= 64) a.xkb = 4, a.xring = 2 * 4 * npad * 128;
+    else if (npad <= 128) a.xkb = 2, a.xring = 2 * 2 * npad * 128;
+  }
+  if (env_xkb > 0) a.xkb = env_xkb;
+  const int nk_all = a.kslice / kBK;
+  if (EPI == EPI_PROJ) {
+    if (a.xkb > 1 && (a.H / kBK) % a.xkb != 0) a.xkb = 1;
+  } else if (nk_all % a.xkb != 0) {
+    a.xkb = 1;
+  }
   const int wblk = (EPI == EPI_PROJ ? 128 : gates_of(EPI) * a.U) * 128;
-  const size_t smem = 1024 + kTailBytes + region_bytes(npad, a.wcb, a.xring, wblk);
+  const size_t smem = 1024 + kTailBytes + region_bytes(npad, a.wcb, a.xring, wblk, a.xkb);
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int S = EPI == EPI_PROJ ? 1 : a.S;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;

@@ -52,7 +52,7 @@ constexpr int kMaxStages = 8;
 // cell kernel. out: per CTA {cycles to first stage, cycles to last stage}; img: CTA 0's stages.
 __global__ void __launch_bounds__(256) gather_kernel(const __grid_constant__ CUtensorMap map,
                                                      const __nv_bfloat16* table, int H, const int* idx,
-                                                     int npad, int nk, int mode, long long* out,
+                                                     int npad, int nk, int mode, long long* out, int rot,
                                                      uint8_t* img, int reps) {
   extern __shared__ __align__(1024) uint8_t sm_raw[];
   uint8_t* sm = (uint8_t*)(((uintptr_t)sm_raw + 1023) & ~(uintptr_t)1023);
@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(256) gather_kernel(const __grid_constant__ CUt
   long long t_first = 0, t_last = 0;
   for (int rep = 0; rep < reps; ++rep) {
     if (tid == 0) {
-      for (int s = 0; s < nk; ++s) mbar_init(su32(&full[s]), 1);
+      for (int s = 0; s < nk; ++s) mbar_init(su32(&full[s]), mode == 3 ? 256 : 1);
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -80,6 +80,53 @@ __global__ void __launch_bounds__(256) gather_kernel(const __grid_constant__ CUt
             gather4(su32(sm + s * stage_bytes + g * 512), &map, s * 64, r.x, r.y, r.z, r.w, su32(&full[s]));
           }
         }
+      }
+    } else if (mode == 2) {
+      // LDG.128 into registers (a batch of stages per thread in flight), STS into the swizzled
+      // stage, proxy fence, block barrier, one arrive per stage
+      if (tid < npad) rows_s[tid] = max(myidx[tid], 0);
+      __syncthreads();
+      const int per = npad * 8 / 256 > 0 ? npad * 8 / 256 : 1;   // items per thread per stage
+      const int batch = per >= 8 ? 2 : (per >= 4 ? 4 : 8);         // stages per batch (<= 16 items)
+      for (int s0 = 0; s0 < nk; s0 += batch) {
+        uint4 v[16];
+        uint32_t dst[16];
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int s = s0 + j / per, i = j % per;
+          const int q = tid + 256 * i;
+          v[j] = make_uint4(0, 0, 0, 0);
+          dst[j] = 0xFFFFFFFFu;
+          if (j < batch * per && s < nk && q < npad * 8) {
+            const int row = q >> 3, ch = q & 7;
+            const uint4* src = reinterpret_cast<const uint4*>(table + (size_t)rows_s[row] * H + s * 64 + ch * 8);
+            asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v[j].x), "=r"(v[j].y), "=r"(v[j].z), "=r"(v[j].w) : "l"(src));
+            dst[j] = su32(sm + s * stage_bytes) + row * 128 + ((ch ^ (row & 7)) << 4);
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < 16; ++j)
+          if (dst[j] != 0xFFFFFFFFu)
+            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(dst[j]), "r"(v[j].x), "r"(v[j].y), "r"(v[j].z), "r"(v[j].w) : "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("bar.sync 1, 256;" ::: "memory");
+        if (tid == 0)
+          for (int s = s0; s < min(nk, s0 + batch); ++s)
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&full[s])) : "memory");
+      }
+    } else if (mode == 3) {
+      // cp.async with one cp.async.mbarrier.arrive.noinc per thread per stage (count 256)
+      if (tid < npad) rows_s[tid] = max(myidx[tid], 0);
+      __syncthreads();
+      for (int s = 0; s < nk; ++s) {
+        const uint32_t xs = su32(sm + s * stage_bytes);
+        for (int q = tid; q < npad * 8; q += 256) {
+          const int row = ((q >> 3) + (rot ? (blockIdx.x / 4) * 8 : 0)) % npad, ch = q & 7;
+          const __nv_bfloat16* src = table + (size_t)rows_s[row] * H + s * 64 + ch * 8;
+          const uint32_t dst = xs + row * 128 + ((ch ^ (row & 7)) << 4);
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+        }
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[s])) : "memory");
       }
     } else {
       if (tid < npad) rows_s[tid] = max(myidx[tid], 0);
@@ -138,7 +185,8 @@ __global__ void __launch_bounds__(256) gather_kernel(const __grid_constant__ CUt
 }
 
 int main(int argc, char** argv) {
-  const int R = 65536, H = 1024;
+  const int R = argc > 2 ? atoi(argv[2]) : 65536, H = 1024;
+  const int share = argc > 3 ? atoi(argv[3]) : 0;
   std::vector<__nv_bfloat16> h((size_t)R * H);
   for (size_t r = 0; r < (size_t)R; ++r)
     for (int c = 0; c < H; ++c) h[r * H + c] = __float2bfloat16((float)((r * 7 + c) % 251));
@@ -170,11 +218,12 @@ int main(int argc, char** argv) {
   for (int npad : {16, 64, 128, 256}) {
     std::vector<int> idx(nsm * 256);
     for (auto& x : idx) x = rand() % R;
+    if (share) for (int c = 0; c < nsm; ++c) for (int r = 0; r < 256; ++r) idx[c * 256 + r] = idx[(c % 4) * 256 + r];
     for (int i = 0; i < 4; ++i) idx[i] = (i == 1) ? -1 : idx[i];  // a negative row: OOB -> zero fill?
     CK(cudaMemcpy(didx, idx.data(), idx.size() * 4, cudaMemcpyHostToDevice));
     const int nk = npad <= 64 ? 8 : (npad == 128 ? 8 : 6);
-    for (int mode = 0; mode < 2; ++mode) {
-      gather_kernel<<<nsm, 256, 200 * 1024>>>(map, d, H, didx, npad, nk, mode, dout, dimg, 20);
+    for (int mode = 3; mode < 4; ++mode) {
+      gather_kernel<<<nsm, 256, 200 * 1024>>>(map, d, H, didx, npad, nk, mode, dout, share == 2, dimg, 20);
       CK(cudaGetLastError());
       CK(cudaDeviceSynchronize());
       std::vector<long long> o(nsm * 2);
@@ -202,7 +251,7 @@ int main(int argc, char** argv) {
       double f = 0, l = 0;
       for (int i = 0; i < nsm; ++i) f += o[2 * i], l += o[2 * i + 1];
       printf("%-8s npad %3d nk %d: first stage %6.0f cyc, all %6.0f cyc (%.2f us @1.9GHz, %.1f GB/s/SM)  bad %d zero-fill %s\n",
-             mode == 0 ? "gather4" : "cp.async", npad, nk, f / nsm, l / nsm, l / nsm / 1900.0,
+             mode == 0 ? "gather4" : mode == 1 ? "cp.async" : mode == 2 ? "ldg+sts" : "cpa+arrv", npad, nk, f / nsm, l / nsm, l / nsm / 1900.0,
              (double)nk * npad * 128 / (l / nsm / 1.9), bad, mode == 0 ? (zero_ok ? "ok" : "NO") : "n/a");
     }
   }
