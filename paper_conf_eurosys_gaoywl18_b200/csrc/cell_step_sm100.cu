@@ -142,13 +142,43 @@ __device__ __forceinline__ void launch_done(const StepArgs& p, unsigned int* cta
 }
 
 // ------------------------------------------------------------------ row sources (A6)
-// Row i of the launch: from the inline parameter block, or from device memory (a.rows).
-__device__ __forceinline__ RowDesc row_at(const StepArgs& p, const StepRows& rr, int i) {
-  if (p.rows != nullptr) {
-    const int4 v = __ldg(reinterpret_cast<const int4*>(p.rows) + i);
+// The launch's rows travel either inline in the parameter block (RowsParam<true>, direct
+// steps) or in the device descriptor ring (RowsParam<false>: a 4-byte dummy, so the launch
+// carries ~0.5 KB of parameters instead of ~8.7 KB -- 3.3 vs 6.5-8.9 us of host time per
+// launch, tools/launch_bench.cu). Ring rows are published by a copy on the copy stream
+// followed by a stream write of rows_seq to *rows_flag; the kernel polls the flag (acquire)
+// before its first row read, so no cross-stream event sits between two launches.
+template <bool INL>
+struct RowsParam {
+  RowDesc r[kMaxRowsInline];
+};
+template <>
+struct RowsParam<false> {
+  int unused;
+};
+template <bool INL>
+__device__ __forceinline__ RowDesc row_at(const StepArgs& p, const RowsParam<INL>& rr, int i) {
+  if constexpr (INL) {
+    return rr.r[i];
+  } else {
+    const int4 v = *(reinterpret_cast<const int4*>(p.rows) + i);
     return RowDesc{v.x, v.y, v.z, v.w};
   }
-  return rr.r[i];
+}
+// Ring rows: wait until the copy that carries them has landed (lane 0 polls, 10 s trap).
+__device__ __forceinline__ void rows_wait(const StepArgs& p) {
+  if (p.rows_flag == nullptr) return;
+  if ((threadIdx.x & 31) == 0) {
+    unsigned long long t0 = 0;
+    while (static_cast<int>(ld_acquire_gpu(p.rows_flag) - p.rows_seq) < 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 10000000000ull) __trap();
+    }
+  }
+  __syncwarp();
+  (void)ld_acquire_gpu(p.rows_flag);
 }
 
 // Pointer to the first element of a row's operand segment `seg`, or nullptr for a zero row.
@@ -180,9 +210,9 @@ __device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const
 }
 
 // ------------------------------------------------------------------ the kernel
-template <int EPI>
+template <int EPI, bool INL>
 __global__ void __launch_bounds__(kThreads, 2)
-    cell_step_sm100_kernel(const __grid_constant__ StepArgs p, const __grid_constant__ StepRows rr) {
+    cell_step_sm100_kernel(const __grid_constant__ StepArgs p, const __grid_constant__ RowsParam<INL> rr) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
@@ -270,6 +300,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     // the launch's own rows (independent of earlier launches) into the smem table: one 16-byte
     // parameter load per thread (parameter loads miss the constant cache and serialise per
     // address: each row is read once and then shared through shared memory)
+    if constexpr (!INL) rows_wait(p);
     if (tid < ncols) rtab[tid] = row_at(p, rr, col0 + tid);
     named_bar(1, kProducerThreads);
 #pragma unroll
@@ -645,8 +676,11 @@ template <int EPI>
 cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   static bool configured = false;
   if (!configured) {
-    cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI>,
+    cudaError_t e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI, true>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(cell_step_sm100_kernel<EPI, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               227 * 1024);
     if (e != cudaSuccess) return e;
     configured = true;
   }
@@ -667,6 +701,7 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   if (!internal && EPI != EPI_LEAF) {
     if (npad <= 64) a.xkb = 4, a.xring = 2 * 4 * npad * 128;
     else if (npad <= 128) a.xkb = 2, a.xring = 2 * 2 * npad * 128;
+    else if (env_wcb == 0) a.xkb = 2, a.wcb = 2, a.xring = 2 * 2 * npad * 128;  // 64 KB weight ring
   }
   if (env_xkb > 0) a.xkb = env_xkb;
   const int nk_all = a.kslice / kBK;
@@ -694,15 +729,16 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   attr[1].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
-  static thread_local StepRows inline_rows;
   if (rows_host != nullptr) {
+    static thread_local RowsParam<true> inline_rows;
     if (a.b > kMaxRowsInline) return cudaErrorInvalidValue;
     memcpy(inline_rows.r, rows_host, sizeof(RowDesc) * a.b);
     a.rows = nullptr;
-  } else if (a.rows == nullptr) {
-    return cudaErrorInvalidValue;
+    a.rows_flag = nullptr;
+    return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI, true>, a, inline_rows);
   }
-  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI>, a, inline_rows);
+  if (a.rows == nullptr) return cudaErrorInvalidValue;
+  return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI, false>, a, RowsParam<false>{0});
 }
 
 }  // namespace

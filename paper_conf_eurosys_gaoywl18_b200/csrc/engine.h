@@ -192,6 +192,12 @@ struct Engine {
   unsigned int* dep_flag = nullptr;  // launch chain flag (device): last completed sm100 launch
   unsigned int dep_seq = 0;          // host: sequence number of the last sm100 launch issued
   bool pdl_ok = false;               // the stream's last op was an sm100 launch (PDL is safe)
+  // ring rows of the tcgen05 path: published by a copy + a flag write on copy_stream
+  unsigned int* rows_flag_dev = nullptr;   // device: last published rows sequence number
+  unsigned int* rows_seq_host = nullptr;   // pinned ring of sequence values (flag-copy fallback)
+  unsigned int rows_seq = 0;               // host: last sequence number issued
+  unsigned int launch_rows_seq = 0;        // 0: the launch's rows need no flag wait
+  void* write_value32 = nullptr;           // cuStreamWriteValue32 (driver entry point) or null
   RowDesc* ring_dev = nullptr;
   RowDesc* ring_host = nullptr;    // pinned staging
   int ring_rows = 0;

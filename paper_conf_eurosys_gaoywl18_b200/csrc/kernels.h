@@ -68,6 +68,8 @@ struct StepArgs {
                               // activation ring bytes, K blocks per activation stage
   unsigned long long* span;   // time_kernels: slot {min CTA start, CTAs done} (device memory)
   unsigned long long* span_acc;  // {sum of launch spans in ns, launches}: last CTA adds
+  const unsigned int* rows_flag;  // ring rows: published once *rows_flag >= rows_seq (or null)
+  unsigned int rows_seq;
   unsigned int* dep_flag;     // launch chain: sequence number of the last completed launch
   unsigned int dep_seq;       // this launch's sequence number (waits for dep_seq - 1)
   unsigned long long* tl;     // diagnostics (BM_TIMELINE): {~first CTA start, ~first past the
@@ -109,9 +111,6 @@ int persistent_smem_bytes();
 // no host->device copy and no cross-stream dependency between consecutive launches, so PDL
 // overlaps a launch's prologue with the previous launch's tail).
 constexpr int kMaxRowsInline = 512;
-struct StepRows {
-  RowDesc r[kMaxRowsInline];
-};
 // rows_host: the launch's rows in host memory (b <= kMaxRowsInline) -- passed inline; or null,
 // then a.rows must point to device memory holding them.
 cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st);

@@ -127,6 +127,10 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
     a.dep_flag = e.dep_flag;
     a.dep_seq = e.dep_seq + 1;
   }
+  if (rows_dev != nullptr && e.launch_rows_seq != 0) {
+    a.rows_flag = e.rows_flag_dev;
+    a.rows_seq = e.launch_rows_seq;
+  }
   TimedLaunch* tl = nullptr;
   // events serialise the stream and so disable PDL overlap around the launches they bracket:
   // time a sample (every kTimeEvery-th launch) instead of every launch
@@ -224,8 +228,9 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
     }
   }
   if (!e.device()) return BM_OK;
-  if (e.cfg.precision == BM_PREC_BF16 && !e.persistent_active) {
-    // tcgen05 path: each launch carries its task's row descriptors as a kernel parameter
+  static const int rows_inline = getenv("BM_ROWS_INLINE") ? atoi(getenv("BM_ROWS_INLINE")) : 0;
+  if (e.cfg.precision == BM_PREC_BF16 && !e.persistent_active && rows_inline) {
+    // diagnostics: each launch carries its task's row descriptors as a kernel parameter
     for (Task& t : tasks) {
       bm_status s = launch_cell(e, e.cells[t.ct], nullptr, t.desc.data(), t.b, &t, e.signal_dev);
       if (s != BM_OK) return s;
@@ -272,11 +277,34 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
                          e.copy_stream));
     return BM_OK;
   }
-  // descriptors travel on the copy stream: the copy overlaps the kernels still running, and the
-  // kernel stream only waits on an event that has usually fired by the time it gets there (an
-  // in-stream copy would sit between two launches, on the critical path, and break PDL)
+  // descriptors travel on the copy stream: the copy overlaps the kernels still running
   CK(cudaMemcpyAsync(e.ring_dev + base, e.ring_host + base, sizeof(RowDesc) * total,
                      cudaMemcpyHostToDevice, e.copy_stream));
+  if (e.cfg.precision == BM_PREC_BF16) {
+    // tcgen05 path: publish the rows with a flag write behind the copy; each launch polls the
+    // flag on the device, so the kernel stream never waits on the copy stream (PDL stays on)
+    const unsigned int seq = ++e.rows_seq;
+    if (e.write_value32 != nullptr) {
+      using WV = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+      if (reinterpret_cast<WV>(e.write_value32)(e.copy_stream, reinterpret_cast<CUdeviceptr>(e.rows_flag_dev),
+                                                seq, 0) != CUDA_SUCCESS)
+        return BM_E_CUDA;
+    } else {
+      unsigned int* v = e.rows_seq_host + (seq % 256);
+      *v = seq;
+      CK(cudaMemcpyAsync(e.rows_flag_dev, v, 4, cudaMemcpyHostToDevice, e.copy_stream));
+    }
+    e.launch_rows_seq = seq;
+    for (Task& t : tasks) {
+      bm_status s = launch_cell(e, e.cells[t.ct], e.ring_dev + t.ring_off, nullptr, t.b, &t, e.signal_dev);
+      if (s != BM_OK) {
+        e.launch_rows_seq = 0;
+        return s;
+      }
+    }
+    e.launch_rows_seq = 0;
+    return BM_OK;
+  }
   CK(cudaEventRecord(e.copy_ev, e.copy_stream));
   CK(cudaStreamWaitEvent(e.stream, e.copy_ev, 0));
   for (Task& t : tasks) {
@@ -469,6 +497,8 @@ static void free_device(Engine& e) {
   if (e.hdr_host) cudaFreeHost(e.hdr_host);
   cudaFree(e.gbar);
   cudaFree(e.perr);
+  cudaFree(e.rows_flag_dev);
+  if (e.rows_seq_host) cudaFreeHost(e.rows_seq_host);
   if (e.stream) cudaStreamDestroy(e.stream);
 }
 
@@ -525,6 +555,19 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
                       cudaHostAllocMapped) != cudaSuccess)
       return fail(BM_E_NOMEM);
     *E.signal_host = 0;
+    // ring-row publication flag (device) + the stream-write entry point (or a pinned value ring)
+    if (dalloc(&E.rows_flag_dev, 1) != cudaSuccess ||
+        cudaHostAlloc(reinterpret_cast<void**>(&E.rows_seq_host), 256 * sizeof(unsigned int),
+                      cudaHostAllocDefault) != cudaSuccess)
+      return fail(BM_E_NOMEM);
+    {
+      cudaDriverEntryPointQueryResult q;
+      void* fn = nullptr;
+      if (!getenv("BM_NO_WRITE_VALUE") &&
+          cudaGetDriverEntryPoint("cuStreamWriteValue32", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+          q == cudaDriverEntryPointSuccess)
+        E.write_value32 = fn;
+    }
     if (cudaHostGetDevicePointer(reinterpret_cast<void**>(&E.signal_dev), E.signal_host, 0) != cudaSuccess)
       return fail(BM_E_CUDA);
     if (cudaMemsetAsync(E.h_pool, 0, L * 2 * S * H * el, E.stream) != cudaSuccess ||
@@ -534,6 +577,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
         cudaMemsetAsync(E.done_ctas, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.sig_ctas, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.dep_flag, 0, 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.rows_flag_dev, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.res_tok, 0, R * c.max_decode_len * 4, E.stream) != cudaSuccess)
       return fail(BM_E_CUDA);
     if (c.time_kernels) {
