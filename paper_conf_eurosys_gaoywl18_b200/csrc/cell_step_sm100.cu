@@ -741,10 +741,532 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   return cudaLaunchKernelEx(&cfg, cell_step_sm100_kernel<EPI, false>, a, RowsParam<false>{0});
 }
 
+// ================================================================== CTA-pair LSTM kernel
+// cell_pair_kernel: the LSTM cell step (A6-A9) with tcgen05.mma.cta_group::2 -- two SMs of a
+// TPC share one M = 256 MMA (each holds its own 128-row weight tile, A operand) and each
+// gathers only HALF of the task's activation rows (B operand, N/2 rows per CTA; the MMA reads
+// both halves), so the per-CTA gather -- the cp.async issue rate bounds it (tools/
+// ldgsts_bench.cu, exp bits of cell_step_sm100_kernel) -- halves for the same weight tile.
+//
+// Grid (2S, tiles/2, column blocks), cluster (2S, 1, 1): cluster rank r = 2s + m, m = pair
+// member (0 = leader: issues the MMAs), s = K slice. Each CTA's TMEM receives its own 128 rows
+// x all N columns, so the epilogue (split-K DSMEM reduction over the S CTAs with the same m,
+// fixed order -> batch invariant) is the single-CTA kernel's.
+//
+// Hand-offs: producers of each CTA arrive on their local `full` barrier; in the peer CTA the
+// (otherwise idle) MMA warp forwards each completed local stage / weight chunk to the leader's
+// pfull / pwfull barriers (remote mbarrier arrive, release.cluster). The leader's commits
+// multicast to both CTAs' `empty` / `wempty` / `done` barriers.
+namespace pairk {
+constexpr int kStagesMax = 4;
+}
+
+__device__ __forceinline__ bool mbar_try_wait_cluster(uint32_t bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(bar), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// Bounded spin on an mbarrier phase (traps after ~4 s instead of hanging the GPU).
+template <bool CLUSTER>
+__device__ __forceinline__ void wait_bounded(uint32_t bar, uint32_t parity) {
+  unsigned long long t0 = 0;
+  for (int it = 0;; ++it) {
+    if (CLUSTER ? mbar_try_wait_cluster(bar, parity) : mbar_try_wait(bar, parity)) return;
+    if ((it & 1023) == 1023) {
+      const unsigned long long t = gtimer();
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 4000000000ull) __trap();
+    }
+  }
+}
+__device__ __forceinline__ void wait_bounded_warp(uint32_t bar, uint32_t parity) {
+  if ((threadIdx.x & 31) == 0) wait_bounded<false>(bar, parity);
+  __syncwarp();
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+__device__ __forceinline__ void mma_bf16_pair(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc,
+                                              uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void mma_commit_pair(uint32_t bar, uint16_t mask) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          bar),
+      "h"(mask)
+      : "memory");
+}
+__device__ __forceinline__ void cluster_arrive() {
+  asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() {
+  asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <bool INL>
+__global__ void __launch_bounds__(kThreads, 1)
+    cell_pair_kernel(const __grid_constant__ StepArgs p, const __grid_constant__ RowsParam<INL> rr) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5;
+  const int lane = tid & 31;
+  constexpr int G = 4;
+  const int U = p.U;                                      // 32 units per 128-row tile
+  const uint32_t crank = cluster_rank();
+  const int pm = static_cast<int>(crank & 1u);            // pair member (0 = leader)
+  const int ks = static_cast<int>(crank >> 1);            // K slice
+  const int tile = 2 * blockIdx.y + pm;
+  const int cpb = p.cpb;                                  // columns per block
+  const int col0 = blockIdx.z * cpb;
+  const int ncols = min(cpb, p.b - col0);
+  const int npad = (ncols + 31) & ~31;                    // MMA N (both halves)
+  const int nhalf = npad >> 1;                            // rows gathered by this CTA
+  const int h0 = pm * nhalf;
+  const int nk = p.kslice / kBK;
+  const int k_begin = ks * p.kslice;
+  const int xkb = p.xkb > 0 ? p.xkb : 1;
+  const int nst = nk / xkb;
+  const int x_blk_bytes = nhalf * 128;
+  const int x_stage_bytes = x_blk_bytes * xkb;
+  const int kStages = min(pairk::kStagesMax, max(2, p.xring / x_stage_bytes));
+  const int wcb = p.wcb;
+  const int kpc = min(wcb, nk);
+  const int n_chunks = (nk + kpc - 1) / kpc;
+  constexpr int wblk_bytes = 128 * 128;
+  const uint16_t pair_mask = static_cast<uint16_t>(3u << (crank & ~1u));
+
+  uint64_t* bars = reinterpret_cast<uint64_t*>(base);
+  const uint32_t full0 = smem_u32(bars);                              // local producers
+  const uint32_t empty0 = smem_u32(bars + pairk::kStagesMax);         // leader commit (multicast)
+  const uint32_t pfull0 = smem_u32(bars + 2 * pairk::kStagesMax);     // peer stage forwarded
+  const uint32_t wfull0 = smem_u32(bars + 3 * pairk::kStagesMax);     // local weight chunk
+  const uint32_t wempty0 = smem_u32(bars + 3 * pairk::kStagesMax + kWRing);
+  const uint32_t pwfull0 = smem_u32(bars + 3 * pairk::kStagesMax + 2 * kWRing);
+  const uint32_t done_bar = smem_u32(bars + 3 * pairk::kStagesMax + 3 * kWRing);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * pairk::kStagesMax + 3 * kWRing + 1);
+  RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);
+  uint8_t* smem = base + kTailBytes;
+  uint8_t* w_ring = smem;
+  uint8_t* x_st = smem + kWRing * wcb * wblk_bytes;
+
+  if (tid == 0) phase_mark(p, 0);
+  if (tid == 0) {
+    for (int s = 0; s < pairk::kStagesMax; ++s) {
+      mbar_init(full0 + 8 * s, kProducerThreads);
+      mbar_init(empty0 + 8 * s, 1);
+      mbar_init(pfull0 + 8 * s, 1);
+    }
+    for (int s = 0; s < kWRing; ++s) {
+      mbar_init(wfull0 + 8 * s, 1);
+      mbar_init(wempty0 + 8 * s, 1);
+      mbar_init(pwfull0 + 8 * s, 1);
+    }
+    mbar_init(done_bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == kMmaWarp) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(256)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  cluster_arrive();  // barrier inits of every CTA visible before any remote arrive / multicast
+  const uint32_t tmem = *tmem_slot;
+  pdl_launch_dependents();
+  if (tid == 0) phase_mark(p, 1);
+
+  if (warp < 8) {
+    // ================================================================ activation gather (A6)
+    constexpr int kItems = 4;  // nhalf <= 128 rows x 8 chunks / 256 threads
+    const int n_items = (nhalf * 8 + kProducerThreads - 1 - tid) / kProducerThreads;
+    if constexpr (!INL) rows_wait(p);
+    if (tid < ncols) rtab[tid] = row_at(p, rr, col0 + tid);
+    named_bar(1, kProducerThreads);
+    const __nv_bfloat16* src0[kItems];
+    const __nv_bfloat16* src1[kItems];
+    uint32_t dst_off[kItems];
+    RowDesc rd[kItems];
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) rd[i] = rtab[min(h0 + ((tid + i * kProducerThreads) >> 3), ncols - 1)];
+    dep_wait(p);
+    if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
+    if (tid == 0) phase_mark(p, 8);
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {
+      const int q = tid + i * kProducerThreads;
+      const int row = q >> 3;
+      const int ch = q & 7;
+      dst_off[i] = row * 128 + ((ch ^ (row & 7)) << 4);
+      src0[i] = nullptr;
+      src1[i] = nullptr;
+      if (i < n_items && h0 + row < ncols) {
+        const __nv_bfloat16* a0 = seg_src<EPI_LSTM>(p, rd[i], 0);
+        const __nv_bfloat16* a1 = seg_src<EPI_LSTM>(p, rd[i], 1);
+        src0[i] = a0 != nullptr ? a0 + ch * 8 : nullptr;
+        src1[i] = a1 != nullptr ? a1 + ch * 8 : nullptr;
+      }
+    }
+    const __nv_bfloat16* dummy = static_cast<const __nv_bfloat16*>(p.E != nullptr ? p.E : p.h_pool);
+    for (int st = 0; st < nst; ++st) {
+      const int s = st % kStages;
+      const int round = st / kStages;
+      if (round > 0) wait_bounded_warp(empty0 + 8 * s, (round - 1) & 1);
+      for (int j = 0; j < xkb; ++j) {
+        const int k = k_begin + (st * xkb + j) * kBK;
+        const int seg = k >= p.K0 ? 1 : 0;
+        const int kk = k - seg * p.K0;
+        const uint32_t xs = smem_u32(x_st + s * x_stage_bytes + j * x_blk_bytes);
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+          if (i < n_items) {
+            const __nv_bfloat16* src = seg ? src1[i] : src0[i];
+            if (src != nullptr) cp_async_16(xs + dst_off[i], src + kk, 16);
+            else cp_async_16(xs + dst_off[i], dummy, 0);  // zero fill (h0 = 0, padding)
+          }
+        }
+      }
+      cp_async_arrive_noinc(full0 + 8 * s);
+      if (tid == 0 && st == 0) phase_mark(p, 10);
+    }
+  } else if (warp == kTmaWarp) {
+    // ================================================================ weight stream (A7)
+    if (lane == 0) {
+      const int kblocks = (p.K0 + p.K1) / kBK;
+      const uint8_t* wsrc =
+          static_cast<const uint8_t*>(p.W) + (static_cast<size_t>(tile) * kblocks + k_begin / kBK) * wblk_bytes;
+      for (int c = 0; c < n_chunks; ++c) {
+        const int s = c % kWRing;
+        const int round = c / kWRing;
+        if (round > 0) wait_bounded<false>(wempty0 + 8 * s, (round - 1) & 1);
+        const int nblk = min(kpc, nk - c * kpc);
+        const uint32_t bytes = static_cast<uint32_t>(nblk * wblk_bytes);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(wfull0 + 8 * s), "r"(bytes)
+                     : "memory");
+        bulk_load(smem_u32(w_ring + s * wcb * wblk_bytes), wsrc + static_cast<size_t>(c) * kpc * wblk_bytes, bytes,
+                  wfull0 + 8 * s);
+      }
+    }
+    __syncwarp();
+  } else if (pm == 0) {
+    // ================================================================ MMA issuer (leader, A8)
+    cluster_wait();
+    const uint32_t idesc = idesc_bf16(256, npad);
+    for (int st = 0; st < nst; ++st) {
+      const int s = st % kStages;
+      const uint32_t par = (st / kStages) & 1;
+      if (lane == 0) {
+        wait_bounded<false>(full0 + 8 * s, par);
+        if (st < 4) phase_mark(p, 40 + st);
+        wait_bounded<true>(pfull0 + 8 * s, par);
+        if (st < 4) phase_mark(p, 44 + st);
+      }
+      __syncwarp();
+      tc_fence_after();
+      if (lane == 0 && st < 12) phase_mark(p, 16 + st);
+      if (lane == 0 && st == 0) phase_mark(p, 6);
+      if (lane == 0 && st == nst - 1) phase_mark(p, 7);
+      for (int j = 0; j < xkb; ++j) {
+        const int kb = st * xkb + j;
+        const int c = kb / kpc;
+        const int ws = c % kWRing;
+        if (kb % kpc == 0) {
+          const uint32_t wpar = (c / kWRing) & 1;
+          if (lane == 0) {
+            wait_bounded<false>(wfull0 + 8 * ws, wpar);
+            if (c < 4) phase_mark(p, 48 + c);
+            wait_bounded<true>(pwfull0 + 8 * ws, wpar);
+            if (c < 4) phase_mark(p, 52 + c);
+          }
+          __syncwarp();
+          tc_fence_after();
+        }
+        if (lane == 0) {
+          const uint64_t a = sdesc_sw128(smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
+          const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes + j * x_blk_bytes));
+#pragma unroll
+          for (int k = 0; k < kBK / 16; ++k) mma_bf16_pair(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
+          if (kb % kpc == kpc - 1 || kb == nk - 1) mma_commit_pair(wempty0 + 8 * ws, pair_mask);
+        }
+        __syncwarp();
+      }
+      if (lane == 0) {
+        mma_commit_pair(empty0 + 8 * s, pair_mask);
+        if (st == nst - 1) mma_commit_pair(done_bar, pair_mask);
+      }
+      __syncwarp();
+    }
+  } else {
+    // ================================================================ forwarder (peer)
+    cluster_wait();
+    const uint32_t lead = crank & ~1u;
+    const uint32_t pfull_l = mapa(pfull0, lead);
+    const uint32_t pwfull_l = mapa(pwfull0, lead);
+    if (lane == 0) {
+      for (int st = 0; st < nst; ++st) {
+        const int s = st % kStages;
+        wait_bounded<false>(full0 + 8 * s, (st / kStages) & 1);
+        if (st < 4) phase_mark(p, 40 + st);
+        fence_proxy_async();
+        mbar_arrive_remote(pfull_l + 8 * s);
+        for (int j = 0; j < xkb; ++j) {
+          const int kb = st * xkb + j;
+          if (kb % kpc == 0) {
+            const int c = kb / kpc;
+            const int ws = c % kWRing;
+            wait_bounded<false>(wfull0 + 8 * ws, (c / kWRing) & 1);
+            if (c < 4) phase_mark(p, 48 + c);
+            mbar_arrive_remote(pwfull_l + 8 * ws);
+          }
+        }
+      }
+    }
+    __syncwarp();
+  }
+  if (warp != kMmaWarp) cluster_wait();
+
+  // ================================================================ epilogue (A9)
+  wait_bounded_warp(done_bar, 0);
+  tc_fence_after();
+  if (tid == 0) phase_mark(p, 2);
+  const int q = warp & 3;
+  const int trow = 32 * q + lane;
+  const int S = p.S;
+  const int cper = (ncols + S - 1) / S;
+  float* P = reinterpret_cast<float*>(smem);
+  constexpr int pitch = 128;
+  if (warp < 8) {
+    for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
+      float v[32];
+      tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
+#pragma unroll
+      for (int i = 0; i < 32; ++i)
+        if (c0 + i < npad) P[(c0 + i) * pitch + trow] = v[i];
+    }
+  }
+  tc_fence_before();
+  cluster_sync();  // A: every CTA's partial tile is in its smem
+  if (tid == 0) phase_mark(p, 3);
+  uint32_t peer[kMaxS];
+#pragma unroll
+  for (int s = 0; s < kMaxS; ++s) peer[s] = mapa(smem_u32(P), static_cast<uint32_t>(2 * (s < S ? s : 0) + pm));
+  const int c_lo = ks * cper;
+  const int my_cols = max(0, min(ncols, c_lo + cper) - c_lo);
+  const int unit0 = tile * U;
+  const int prow0 = tile * 128;
+  const size_t H = p.H;
+  const size_t NS = p.n_slots;
+  {
+    const int ew = kThreads / U;
+    const int j = tid % U;
+    const int u = unit0 + j;
+    const float4 bias = *reinterpret_cast<const float4*>(p.bias + prow0 + j * G);
+    for (int cl = tid / U; cl < my_cols; cl += 2 * ew) {
+      const int nit = (cl + ew < my_cols) ? 2 : 1;
+      float4 v[2][kMaxS];
+      RowDesc r[2];
+      float cin[2];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (h < nit) {
+          const uint32_t off = static_cast<uint32_t>(((c_lo + cl + h * ew) * pitch + j * G) * 4);
+#pragma unroll
+          for (int s = 0; s < kMaxS; ++s)
+            if (s < S) v[h][s] = ld_cluster_v4(peer[s] + off);
+          r[h] = rtab[c_lo + cl + h * ew];
+          cin[h] = (r[h].flags & ROW_FIRST) ? 0.f : p.c_pool[r[h].slot * H + u];
+        }
+      }
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (h < nit) {
+          float z0 = bias.x, z1 = bias.y, z2 = bias.z, z3 = bias.w;
+#pragma unroll
+          for (int s = 0; s < kMaxS; ++s)  // fixed order s = 0..S-1 (batch invariance)
+            if (s < S) {
+              z0 += v[h][s].x;
+              z1 += v[h][s].y;
+              z2 += v[h][s].z;
+              z3 += v[h][s].w;
+            }
+          const float cn = sigm(z1) * cin[h] + sigm(z0) * tanh_f(z2);
+          const float hn = sigm(z3) * tanh_f(cn);
+          const RowDesc& rw = r[h];
+          p.c_pool[rw.slot * H + u] = cn;
+          const int par_out = (rw.flags & ROW_PARITY) ? 0 : 1;
+          static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + rw.slot) * H + u] = __float2bfloat16_rn(hn);
+          if (rw.flags & ROW_LAST) {
+            const size_t ro = (static_cast<size_t>(rw.flags >> 8) * p.res_layers + p.layer) * H + u;
+            p.res_h[ro] = hn;
+            p.res_c[ro] = cn;
+          }
+        }
+      }
+    }
+  }
+  if (tid == 0) phase_mark(p, 4);
+  tc_fence_before();
+  cluster_sync();  // B: peers may read this CTA's partials until here; both pair TMEMs drained
+  if (tid == 0) phase_mark(p, 5);
+  if (p.dep_flag != nullptr || p.signal != nullptr) {
+    __threadfence();
+    __syncthreads();
+    launch_done(p, p.sig_ctas);
+  }
+  if (warp == kMmaWarp) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256) : "memory");
+  }
+  if (p.span != nullptr) {
+    __syncthreads();
+    if (tid == 0) {
+      __threadfence();
+      const unsigned long long total = gridDim.x * gridDim.y * gridDim.z;
+      if (atomicAdd(p.span + 1, 1ull) == total - 1) {
+        const unsigned long long t0 = atomicExch(p.span, ~0ull);
+        atomicExch(p.span + 1, 0ull);
+        atomicAdd(p.span_acc, gtimer() - t0);
+        atomicAdd(p.span_acc + 1, 1ull);
+      }
+    }
+  }
+}
+
+// Launch plan of the pair kernel; returns false if the task is not eligible (caller falls back).
+// S = 4 (512-wide K slices, clusters of 8) for small tasks when 16 such clusters are
+// co-resident, else S = 2 (1024-wide slices, clusters of 4); column blocks of <= 256 so a
+// task runs as <= 2 blocks (<= 128 CTAs, one wave).
+template <bool INL>
+cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, bool* done) {
+  *done = false;
+  static int state = 0;  // 0 unknown, 1 usable, -1 not usable
+  static int max_clusters8 = 0;
+  const int smem = 227 * 1024;
+  if (state == 0) {
+    cudaError_t e = cudaFuncSetAttribute(cell_pair_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(cell_pair_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) {
+      state = -1;
+      cudaGetLastError();
+      return cudaSuccess;
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(8, 16, 1);
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = smem;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 8;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    if (cudaOccupancyMaxActiveClusters(&max_clusters8, cell_pair_kernel<false>, &cfg) != cudaSuccess) {
+      max_clusters8 = 0;
+      cudaGetLastError();
+    }
+    state = 1;
+  }
+  if (state < 0) return cudaSuccess;
+  const int K = a.K0 + a.K1;
+  const int tiles = a.H / a.U;
+  // measured (tools/pair_sweep.sh, kbench spans): the pair kernel wins above 256 rows (b = 384:
+  // 23.3 vs 25.7 us) and loses below (b = 64: 17 vs 12 us) -- BM_PAIR_MIN overrides the cut
+  static const int min_b = getenv("BM_PAIR_MIN") ? atoi(getenv("BM_PAIR_MIN")) : 257;
+  if (a.epi != EPI_LSTM || a.U != 32 || tiles % 2 != 0 || K % 1024 != 0 || a.b > 512 || a.b < min_b)
+    return cudaSuccess;
+  static const int env_s = getenv("BM_PAIR_S") ? atoi(getenv("BM_PAIR_S")) : 0;
+  int S = (a.b <= 128 && max_clusters8 >= tiles / 2) ? 4 : 2;
+  if (env_s == 2 || env_s == 4) S = env_s;
+  if (S == 4 && max_clusters8 < tiles / 2) S = 2;
+  if (K / S > 1024 || (K / S) % 256 != 0) return cudaSuccess;
+  a.S = S;
+  a.kslice = K / S;
+  // column blocks: two blocks when that keeps one wave (tiles/2 x 2S x blocks <= 148 CTAs)
+  const int ctas1 = (tiles / 2) * 2 * S;
+  int nblk = (ctas1 * 2 <= 148 && a.b > 32) ? 2 : 1;
+  if (a.b > 256) nblk = 2;
+  int cpb = ((a.b + nblk - 1) / nblk + 31) & ~31;
+  if (cpb > 256) return cudaSuccess;
+  nblk = (a.b + cpb - 1) / cpb;
+  if (ctas1 * nblk > 148) return cudaSuccess;
+  a.cpb = cpb;
+  const int nhalf = cpb / 2;
+  const int nk = a.kslice / kBK;
+  // rings: weights 2 x 32 KB (or the whole 128 KB slice when it fits), activations up to 4
+  // stages of xkb K blocks
+  static const int env_wcb = getenv("BM_PAIR_WCB") ? atoi(getenv("BM_PAIR_WCB")) : 0;
+  static const int env_xkb = getenv("BM_PAIR_XKB") ? atoi(getenv("BM_PAIR_XKB")) : 0;
+  a.wcb = 2;
+  a.xkb = env_xkb > 0 ? env_xkb : 4;
+  while (a.xkb > 1 && nk % a.xkb != 0) a.xkb >>= 1;
+  int xstage = nhalf * 128 * a.xkb;
+  const int budget = smem - 1024 - kTailBytes;
+  if (nk * 16 * 1024 + 2 * xstage <= budget && nk <= 8) a.wcb = nk / 2;  // whole slice resident
+  if (env_wcb > 0) a.wcb = env_wcb;
+  int stages = (budget - kWRing * a.wcb * 16 * 1024) / xstage;
+  stages = stages > pairk::kStagesMax ? pairk::kStagesMax : stages;
+  if (stages < 2) return cudaSuccess;
+  a.xring = stages * xstage;
+  const int region = kWRing * a.wcb * 16 * 1024 + a.xring;
+  const int pbytes = cpb * 128 * 4;
+  const size_t need = 1024 + kTailBytes + (region > pbytes ? region : pbytes);
+  if (need > static_cast<size_t>(smem)) return cudaSuccess;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(2 * S, tiles / 2, nblk);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = need;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2 * S;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 2;
+  *done = true;
+  if constexpr (INL) {
+    static thread_local RowsParam<true> inline_rows;
+    memcpy(inline_rows.r, rows_host, sizeof(RowDesc) * a.b);
+    a.rows = nullptr;
+    a.rows_flag = nullptr;
+    return cudaLaunchKernelEx(&cfg, cell_pair_kernel<true>, a, inline_rows);
+  } else {
+    return cudaLaunchKernelEx(&cfg, cell_pair_kernel<false>, a, RowsParam<false>{0});
+  }
+}
+
 }  // namespace
 
 cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st) {
   if (a.b <= 0) return cudaSuccess;
+  static const int use_pair = getenv("BM_PAIR") ? atoi(getenv("BM_PAIR")) : 1;
+  if (use_pair && a.epi == EPI_LSTM) {  // CTA-pair path (falls through if not eligible)
+    bool done = false;
+    cudaError_t e = rows_host != nullptr ? (a.b <= kMaxRowsInline ? launch_pair<true>(a, rows_host, st, &done)
+                                                                   : cudaSuccess)
+                                         : launch_pair<false>(a, rows_host, st, &done);
+    if (done || e != cudaSuccess) return e;
+  }
   switch (a.epi) {
     case EPI_LSTM: return launch_impl<EPI_LSTM>(a, rows_host, st);
     case EPI_LEAF: return launch_impl<EPI_LEAF>(a, rows_host, st);

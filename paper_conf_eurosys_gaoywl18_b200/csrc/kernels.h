@@ -64,6 +64,7 @@ struct StepArgs {
   unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
   unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)
   int pdl;                    // launch with programmatic dependent launch (overlap setup)
+  int cpb;                    // CTA-pair kernel: batch columns per column block
   int wcb, xring, xkb;        // ring plan (set by the launcher): K blocks per weight chunk,
                               // activation ring bytes, K blocks per activation stage
   unsigned long long* span;   // time_kernels: slot {min CTA start, CTAs done} (device memory)

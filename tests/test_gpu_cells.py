@@ -157,3 +157,36 @@ def test_batch_invariance_bitwise(b):
     one_h, one_c = e.result_rows([4000])
     assert np.array_equal(one_h[0], full_h[0])
     assert np.array_equal(one_c[0], full_c[0])
+
+
+@pytest.mark.parametrize("b_small,b_big", [(260, 512), (300, 384)])
+def test_batch_invariance_pair_regime(b_small, b_big):
+    """P10 for the CTA-pair kernel (tasks of 257..512 rows, tcgen05.mma.cta_group::2, S = 2): a
+    row's result is bitwise identical in a task of b_small and of b_big rows (the column block
+    and pair half it lands in differ; its K-order and split-K order do not)."""
+    rng = np.random.default_rng(12)
+    h, V = 1024, 256
+    e, cid, w = lstm_engine(h, 1, V, bm.PREC_BF16)
+    slots = _slots(rng, b_big, 4096)
+    h0 = bf16_vals(rng.uniform(-1, 1, (b_big, h)), bm.PREC_BF16)
+    c0 = rng.uniform(-1, 1, (b_big, h)).astype(np.float32)
+    toks = rng.integers(3, V, size=b_big)
+    flags = bm.ROW_LAST | (np.arange(b_big) << 8)
+    rows = np.stack([toks, np.zeros(b_big), slots, flags], 1)
+    e.pool_write(0, 0, slots, h0, c0)
+    e.cell_step(cid, rows)
+    big_h, big_c = e.result_rows(np.arange(b_big))
+    # the same first rows again, now the LAST b_small rows of a smaller task (other columns)
+    sel = np.concatenate([np.arange(b_small - 40, b_small), np.arange(0, b_small - 40)])
+    e.pool_write(0, 0, slots, h0, c0)
+    e.cell_step(cid, rows[sel])
+    small_h, small_c = e.result_rows(np.arange(b_big)[sel])
+    assert np.array_equal(small_h, big_h[sel])
+    assert np.array_equal(small_c, big_c[sel])
+    # and within tolerance of the oracle
+    for i in (0, b_small - 1):
+        hs, cs = cells.lstm_cell(w.W[0].astype(np.float64), w.b[0].astype(np.float64),
+                                 w.E[toks[i]].astype(np.float64), h0[i].astype(np.float64),
+                                 c0[i].astype(np.float64))
+        assert np.max(np.abs(big_h[i] - hs)) <= STEP_TOL[bm.PREC_BF16]
+        assert np.max(np.abs(big_c[i] - cs)) <= STEP_TOL[bm.PREC_BF16]

@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(256) gather_kernel(const __grid_constant__ CUt
   long long t_first = 0, t_last = 0;
   for (int rep = 0; rep < reps; ++rep) {
     if (tid == 0) {
-      for (int s = 0; s < nk; ++s) mbar_init(su32(&full[s]), mode == 3 ? 256 : 1);
+      for (int s = 0; s < nk; ++s) mbar_init(su32(&full[s]), (mode == 3 || mode == 4) ? 256 : 1);
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -113,6 +113,60 @@ __global__ void __launch_bounds__(256) gather_kernel(const __grid_constant__ CUt
         if (tid == 0)
           for (int s = s0; s < min(nk, s0 + batch); ++s)
             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&full[s])) : "memory");
+      }
+    } else if (mode == 5 || mode == 6) {
+      // mode 5: every stage's copies issued back to back, ONE commit group, wait_group 0,
+      // then the hand-offs (no arrive.noinc between the copies)
+      // mode 6: per-stage commit groups, hand-off of stage s after wait_group(nk-1-s)
+      if (tid < npad) rows_s[tid] = max(myidx[tid], 0);
+      __syncthreads();
+      for (int s = 0; s < nk; ++s) {
+        const uint32_t xs = su32(sm + s * stage_bytes);
+        for (int q = tid; q < npad * 8; q += 256) {
+          const int row = q >> 3, ch = q & 7;
+          const __nv_bfloat16* src = table + (size_t)rows_s[row] * H + s * 64 + ch * 8;
+          const uint32_t dst = xs + row * 128 + ((ch ^ (row & 7)) << 4);
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+        }
+        if (mode == 6) asm volatile("cp.async.commit_group;" ::: "memory");
+      }
+      if (mode == 5) {
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+        asm volatile("bar.sync 1, 256;" ::: "memory");
+        if (tid == 0)
+          for (int s = 0; s < nk; ++s) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&full[s])) : "memory");
+      } else {
+        for (int d = 0; d < nk; ++d) {
+          switch (nk - 1 - d) {
+            case 0: asm volatile("cp.async.wait_group 0;" ::: "memory"); break;
+            case 1: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
+            case 2: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
+            case 3: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
+            case 4: asm volatile("cp.async.wait_group 4;" ::: "memory"); break;
+            case 5: asm volatile("cp.async.wait_group 5;" ::: "memory"); break;
+            case 6: asm volatile("cp.async.wait_group 6;" ::: "memory"); break;
+            default: asm volatile("cp.async.wait_group 7;" ::: "memory"); break;
+          }
+          asm volatile("bar.sync 1, 256;" ::: "memory");
+          if (tid == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&full[d])) : "memory");
+        }
+      }
+    } else if (mode == 4) {
+      // one warp op = one row x 4 consecutive K blocks (512 contiguous bytes); stages in
+      // groups of 4 K blocks, one arrive.noinc per group on each of its 4 barriers
+      if (tid < npad) rows_s[tid] = max(myidx[tid], 0);
+      __syncthreads();
+      for (int s0 = 0; s0 < nk; s0 += 4) {
+        const int g = min(4, nk - s0);
+        for (int q = tid; q < npad * 8 * g; q += 256) {
+          const int row = q / (8 * g), j = q % (8 * g), blk = j >> 3, ch = j & 7;
+          const __nv_bfloat16* src = table + (size_t)rows_s[row] * H + (s0 + blk) * 64 + ch * 8;
+          const uint32_t dst = su32(sm + (s0 + blk) * stage_bytes) + row * 128 + ((ch ^ (row & 7)) << 4);
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+        }
+        for (int b = 0; b < g; ++b)
+          asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[s0 + b])) : "memory");
       }
     } else if (mode == 3) {
       // cp.async with one cp.async.mbarrier.arrive.noinc per thread per stage (count 256)
@@ -222,7 +276,7 @@ int main(int argc, char** argv) {
     for (int i = 0; i < 4; ++i) idx[i] = (i == 1) ? -1 : idx[i];  // a negative row: OOB -> zero fill?
     CK(cudaMemcpy(didx, idx.data(), idx.size() * 4, cudaMemcpyHostToDevice));
     const int nk = npad <= 64 ? 8 : (npad == 128 ? 8 : 6);
-    for (int mode = 3; mode < 4; ++mode) {
+    for (int mode : {3}) {
       gather_kernel<<<nsm, 256, 200 * 1024>>>(map, d, H, didx, npad, nk, mode, dout, share == 2, dimg, 20);
       CK(cudaGetLastError());
       CK(cudaDeviceSynchronize());
@@ -251,7 +305,7 @@ int main(int argc, char** argv) {
       double f = 0, l = 0;
       for (int i = 0; i < nsm; ++i) f += o[2 * i], l += o[2 * i + 1];
       printf("%-8s npad %3d nk %d: first stage %6.0f cyc, all %6.0f cyc (%.2f us @1.9GHz, %.1f GB/s/SM)  bad %d zero-fill %s\n",
-             mode == 0 ? "gather4" : mode == 1 ? "cp.async" : mode == 2 ? "ldg+sts" : "cpa+arrv", npad, nk, f / nsm, l / nsm, l / nsm / 1900.0,
+             mode == 0 ? "gather4" : mode == 1 ? "cp.async" : mode == 2 ? "ldg+sts" : mode == 3 ? "cpa+arrv" : mode == 4 ? "cpa-row4" : mode == 5 ? "cpa-1grp" : "cpa-grps", npad, nk, f / nsm, l / nsm, l / nsm / 1900.0,
              (double)nk * npad * 128 / (l / nsm / 1.9), bad, mode == 0 ? (zero_ok ? "ok" : "NO") : "n/a");
     }
   }
