@@ -67,6 +67,10 @@ def parse():
     p.add_argument("--persistent", type=int, default=-1,
                    help="1: persistent weight-stationary LSTM kernel (configs[1]); 0: one launch per "
                         "task; -1: per-workload default")
+    p.add_argument("--policy", default="cellular", choices=["cellular", "graph"],
+                   help="graph: the padding + bucketing graph-batching baseline of §7.1 (L427: bucket "
+                        "width 10, round robin over buckets) on the same kernels (lstm workload only)")
+    p.add_argument("--bucket-width", type=int, default=10)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--out", default="")
@@ -121,11 +125,13 @@ def weight_arrays(w):
 
 
 # ------------------------------------------------------------------------------ engine
-def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, keep=0, persistent=0):
+def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, keep=0, persistent=0,
+                 policy=0, bucket_width=10):
     h, L, V = WL[wl]["hidden"], WL[wl]["layers"], WL[wl]["vocab"]
     e = bm.Engine(device=device, hidden=h, pool_layers=L, max_slots=1 << 16, max_requests=max_requests,
                   schedule_when_outstanding_leq=lookahead, time_kernels=time_kernels, keep_results=keep,
-                  max_decode_len=340, record_log=0, persistent=persistent)
+                  max_decode_len=340, record_log=0, persistent=persistent, policy=policy,
+                  bucket_width=bucket_width)
     if wl == "lstm":
         c = w["cell"]
         cid = e.load_cell(bm.CELL_LSTM, L, V, 512, 0, c.W, c.b, c.E)
@@ -307,12 +313,17 @@ def main():
         a.lookahead = WL[wl]["lookahead"]
     if a.persistent < 0:
         a.persistent = WL[wl]["persistent"]
+    policy = bm.POLICY_GRAPH if a.policy == "graph" else bm.POLICY_CELLULAR
+    if policy == bm.POLICY_GRAPH and wl != "lstm":
+        raise SystemExit("--policy graph: chain LSTM workload only (reading G5)")
+    if policy == bm.POLICY_GRAPH:
+        a.persistent = 0
     # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink), never again
     w = make_weights(wl)
     if dist is not None:
         shard.broadcast_arrays(weight_arrays(w), dist, device=torch.device("cuda", local))
     e, cells = build_engine(bm, wl, w, local, max_requests=max(n_req, 1 << 15) + 64, lookahead=a.lookahead,
-                            persistent=a.persistent)
+                            persistent=a.persistent, policy=policy, bucket_width=a.bucket_width)
     stream = torch.cuda.ExternalStream(e.stream(), device=torch.device("cuda", local))
 
     def barrier():
@@ -390,7 +401,8 @@ def main():
     # ---- e2e: public API with host buffers (submit from host, descriptors H2D every Schedule
     #      call inside bm_run, final h rows D2H), timed on the host clock around the whole thing
     e2, cells2 = build_engine(bm, wl, w, local, max_requests=n_req + 64, lookahead=a.lookahead,
-                              time_kernels=0, keep=1, persistent=a.persistent)
+                              time_kernels=0, keep=1, persistent=a.persistent, policy=policy,
+                              bucket_width=a.bucket_width)
     L, H = WL[wl]["layers"], WL[wl]["hidden"]
     hbuf = torch.empty((n_req, L, H), dtype=torch.float32).pin_memory().numpy()
     prep2 = e2.prepare_requests(trace, cells2)
@@ -451,7 +463,10 @@ def main():
                            "saturation_burst_rate_per_gpu": mu, "lookahead_k": a.lookahead,
                            "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
                                  "step (serving)", "parallelism": f"request-sharded x{world}",
-                           "persistent_kernel": bool(a.persistent)},
+                           "persistent_kernel": bool(a.persistent),
+                           "policy": ("cellular batching (Algorithm 1)" if policy == bm.POLICY_CELLULAR else
+                                      f"graph-batching baseline: padding + bucketing, width {a.bucket_width}, "
+                                      "round robin over buckets (L427)")},
                 "latency_ms": {"p50": p50 * 1e3, "p90": p90 * 1e3, "p99": p99 * 1e3},
                 "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu,
                 "clocks": clk.summary(), "gpu_launches": int(st["kernel_launches"]),

@@ -83,11 +83,22 @@ typedef struct {
                              /* weight slice stays in shared memory; tasks arrive through */
                              /* a device ring; a grid barrier separates tasks). Ignored   */
                              /* (regular launches) when the engine is not eligible.       */
+  int policy;                /* BM_POLICY_*: cellular batching (Algorithm 1, default) or  */
+                             /* the padding + bucketing graph-batching baseline (§7.1,    */
+                             /* L427-L437; chain requests only)                            */
+  int bucket_width;          /* graph batching: bucket i holds lengths (i*w, (i+1)*w] and */
+                             /* its graph is unrolled to (i+1)*w steps (L427, L631); 10    */
 } bm_config;
+
+enum {
+  BM_POLICY_CELLULAR = 0,    /* Algorithm 1 (L345-L369): requests join / leave between cells */
+  BM_POLICY_GRAPH = 1        /* padding + bucketing, round robin over buckets, a batch runs */
+                             /* its whole padded graph and returns all outputs at its end  */
+};
 
 /* Fill *cfg with defaults: device 0, BF16, WALL, hidden 1024, 1 layer, 65536 slots,
  * 65536 requests, MaxTasksToSubmit 5, Min 1, k 0, max_decode_len 512, keep_results 0,
- * record_log 1, persistent 0. */
+ * record_log 1, persistent 0, policy BM_POLICY_CELLULAR, bucket_width 10. */
 void bm_config_default(bm_config* cfg);
 
 /* ---------------------------------------------------------------- cells (bm_load_cell) */

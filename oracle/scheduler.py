@@ -407,3 +407,116 @@ def replay_requests(reqs, cells_for_kind, **kw) -> Replay:
             d["decode_len"] = q.decode_len
         qs.append(d)
     return rp.run(qs)
+
+
+# ====================================================================== graph batching (N4)
+class GraphBatchingReplay:
+    """The padding + bucketing baseline the paper compares against (MXNet / TensorFlow, §7.1
+    "Bucketing optimization"), as a scheduling policy over the same cell
+    kernels, driven in virtual time like `Replay` (one tick per task, S21 event order).
+
+    Followed from the text:
+      * a request is assigned to a bucket by its length; bucket i handles lengths in
+        (i*W, (i+1)*W], W = bucket width, default 10 (L427)
+      * a dataflow graph is materialised per bucket, i.e. unrolled to (i+1)*W steps: a request
+        of length 21 is padded to 30 (L427, L631)  [reading G2]
+      * round-robin scheduling across buckets (L427); no timeout: a batch starts, even if not
+        full, as soon as a GPU worker is idle and it is the bucket's turn (L433); bmax caps it
+      * the whole graph runs as one unit and returns every output at its end (graph batching:
+        requests cannot join or leave a running batch, L489, L631)
+    Readings where the text is silent (G1-G5):
+      G1 round robin = scan buckets cyclically starting after the last bucket served; requests
+         within a bucket FIFO by admission
+      G2 padded steps run on the pad token (0); a request's result row is its real last step
+      G3 one slot per request (lowest free index, as S22), taken at batch start, freed when the
+         batch completes
+      G4 "idle" = outstanding tasks <= k (as S19); the batch's (i+1)*W step tasks are submitted
+         together, in step order
+      G5 chain requests only (the paper uses padding for LSTM / Seq2Seq and compares TreeLSTM
+         against graph-merging systems instead)
+    """
+
+    def __init__(self, bmax: int, max_slots: int = 1 << 20, bucket_width: int = 10,
+                 schedule_when_outstanding_leq: int = 0):
+        self.bmax, self.W, self.k = bmax, bucket_width, schedule_when_outstanding_leq
+        self.pool = SlotPool(max_slots)
+        self.buckets: Dict[int, deque] = {}
+        self.last_bucket = -1
+        self.lengths: List[int] = []
+        self.tasks: List[Task] = []
+        self.inflight: deque = deque()
+        self.completions: List[Tuple[int, float]] = []
+        self.now = 0.0
+        self.last_finish = 0.0
+        self.batch_of_task: Dict[int, Tuple[List[int], List[int]]] = {}   # last task -> (rids, slots)
+
+    def bucket(self, length: int) -> int:
+        return (length - 1) // self.W          # lengths (i*W, (i+1)*W] -> i
+
+    def admit(self, length: int) -> int:
+        rid = len(self.lengths)
+        self.lengths.append(length)
+        self.buckets.setdefault(self.bucket(length), deque()).append(rid)
+        return rid
+
+    def schedule(self) -> List[Task]:
+        live = sorted(i for i, q in self.buckets.items() if q)
+        if not live:
+            return []
+        nxt = [i for i in live if i > self.last_bucket]
+        i = nxt[0] if nxt else live[0]          # G1: cyclic scan after the last bucket served
+        q = self.buckets[i]
+        n = min(self.bmax, len(q), self.pool.available())
+        if n == 0:
+            return []
+        rids = [q.popleft() for _ in range(n)]
+        self.last_bucket = i
+        slots = [self.pool.alloc() for _ in rids]   # G3
+        steps = (i + 1) * self.W                    # the bucket's unrolled graph
+        out = []
+        for s in range(steps):
+            t = Task(len(self.tasks), 0, 0, self.now, [TaskRow(r, s, sl) for r, sl in zip(rids, slots)])
+            self.tasks.append(t)
+            out.append(t)
+        self.batch_of_task[out[-1].index] = (rids, slots)
+        return out
+
+    def retire(self, task: Task):
+        done = self.batch_of_task.pop(task.index, None)
+        if done is not None:                        # the graph returns all outputs at its end
+            rids, slots = done
+            for r in rids:
+                self.completions.append((r, self.now))
+            for s in sorted(slots):
+                self.pool.release(s)
+
+    def run(self, requests: Sequence[dict], max_ticks: float = 1e9):
+        """requests: dicts with keys arrival, length (chain). Admission order = list order."""
+        pending = list(range(len(requests)))
+        t = 0.0
+        while True:
+            self.now = t
+            while self.inflight and self.inflight[0].finish <= t:
+                self.retire(self.inflight.popleft())
+            while pending and requests[pending[0]]["arrival"] <= t:
+                i = pending.pop(0)
+                self.admit(requests[i]["length"])
+            if len(self.inflight) <= self.k:
+                for task in self.schedule():
+                    start = max(t, self.last_finish)
+                    task.finish = start + 1
+                    self.last_finish = task.finish
+                    self.inflight.append(task)
+            cand = []
+            if self.inflight:
+                cand.append(self.inflight[0].finish)
+            if pending:
+                cand.append(requests[pending[0]]["arrival"])
+            if not cand:
+                break
+            nt = min(cand)
+            assert nt > t
+            t = nt
+            if t > max_ticks:
+                raise RuntimeError("replay did not terminate")
+        return self

@@ -27,6 +27,7 @@ PREC_BF16, PREC_FP32 = 0, 1
 CLOCK_WALL, CLOCK_VIRTUAL, CLOCK_DRY = 0, 1, 2
 CELL_LSTM, CELL_LSTM_PROJ, CELL_TREE_LEAF, CELL_TREE_INTERNAL = 0, 1, 2, 3
 REQ_CHAIN, REQ_SEQ2SEQ, REQ_TREE = 0, 1, 2
+POLICY_CELLULAR, POLICY_GRAPH = 0, 1
 ROW_FIRST, ROW_LAST, ROW_PARITY = 1, 2, 4
 
 
@@ -35,7 +36,7 @@ class Config(C.Structure):
         "device", "precision", "clock", "hidden", "pool_layers", "max_slots", "max_requests",
         "max_tasks_to_submit", "min_followon_batch", "schedule_when_outstanding_leq",
         "max_decode_len", "keep_results", "record_logits", "time_kernels", "record_log",
-        "persistent")]
+        "persistent", "policy", "bucket_width")]
 
 
 class CellDesc(C.Structure):

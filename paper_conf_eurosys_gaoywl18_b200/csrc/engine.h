@@ -147,6 +147,7 @@ struct Task {
   std::vector<TaskRow> rows;
   std::vector<RowDesc> desc; // device row descriptors, built at submission (A3)
   int ev_first = -1, ev_count = 0;  // timed launches (time_kernels)
+  std::vector<int> batch_reqs;      // graph batching: the batch's requests (on its last task)
 };
 
 struct TimedLaunch {
@@ -164,6 +165,8 @@ struct Engine {
   int n_live_reqs = 0;
   uint64_t next_req_id = 0;
   std::deque<int> pending;          // request table indices not yet admitted (FIFO, S21)
+  std::vector<std::deque<int>> buckets;  // graph batching: admitted requests per bucket [G1]
+  int last_bucket = -1;                  // graph batching: round-robin position
   std::vector<int> free_slots_heap; // min-heap of free slots (A4)
   std::deque<Task> inflight;        // in-progress queue (L331, L395)
   uint64_t launched = 0;            // tasks launched so far (== signal target)

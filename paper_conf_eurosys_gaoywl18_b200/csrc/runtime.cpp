@@ -438,6 +438,8 @@ void bm_config_default(bm_config* c) {
   c->time_kernels = 0;
   c->record_log = 1;
   c->persistent = 0;
+  c->policy = BM_POLICY_CELLULAR;
+  c->bucket_width = 10;
 }
 
 static void dump_timeline(Engine& e) {
@@ -508,7 +510,8 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
   if (c.hidden <= 0 || c.hidden % 64 != 0 || c.pool_layers < 1 || c.pool_layers > 8 ||
       c.max_slots < 1 || c.max_requests < 1 || c.max_requests >= (1 << 23) ||
       c.max_tasks_to_submit < 1 || c.min_followon_batch < 1 || c.schedule_when_outstanding_leq < 0 ||
-      c.max_decode_len < 1 || c.precision < 0 || c.precision > 1 || c.clock < 0 || c.clock > 2)
+      c.max_decode_len < 1 || c.precision < 0 || c.precision > 1 || c.clock < 0 || c.clock > 2 ||
+      c.policy < 0 || c.policy > 1 || c.bucket_width < 1)
     return BM_E_INVAL;
   Engine* e = new (std::nothrow) Engine();
   if (e == nullptr) return BM_E_NOMEM;
@@ -740,6 +743,7 @@ bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
     return id >= 0 && id < nc && (e.cells[id].d.kind == k1 || e.cells[id].d.kind == k2);
   };
   if (q->n < 1 || q->tokens == nullptr) return BM_E_INVAL;
+  if (e.cfg.policy == BM_POLICY_GRAPH && q->kind != BM_REQ_CHAIN) return BM_E_INVAL;  // [G5]
   int vocab = 0;
   if (q->kind == BM_REQ_CHAIN) {
     if (!cell_ok(q->cell0, BM_CELL_LSTM, BM_CELL_LSTM)) return BM_E_INVAL;

@@ -98,6 +98,8 @@ void slot_release(Engine& e, int s) {
 }
 
 bool has_ready(const Engine& e) {
+  for (const auto& q : e.buckets)
+    if (!q.empty()) return true;
   for (const Cell& c : e.cells)
     if (c.ready_nodes > 0) return true;
   return false;
@@ -111,6 +113,12 @@ bm_status admit_request(Engine& e, int ri) {
   r.slot = -1;
   r.t_first = -1;
   r.t_done = -1;
+  if (e.cfg.policy == BM_POLICY_GRAPH) {  // padding + bucketing: bucket (i*w, (i+1)*w] (L427)
+    const size_t i = static_cast<size_t>((r.n_nodes - 1) / e.cfg.bucket_width);
+    if (e.buckets.size() <= i) e.buckets.resize(i + 1);
+    e.buckets[i].push_back(ri);
+    return BM_OK;
+  }
   if (r.kind == BM_REQ_CHAIN || r.kind == BM_REQ_SEQ2SEQ) {
     const int S = r.kind == BM_REQ_CHAIN ? r.n_nodes : r.enc_len;
     r.sg2[0] = Subgraph();
@@ -319,9 +327,69 @@ int batch_tasks(Engine& e, int ct, int worker, std::vector<Task>& out) {
 
 }  // namespace
 
+// ---------------------------------------------------------------- graph batching (N4)
+// The padding + bucketing baseline of §7.1 (L427-L437) over the same cell kernels: round robin
+// over non-empty buckets [G1], a batch of <= bmax requests of one bucket runs the bucket's
+// graph unrolled to (i+1)*w steps -- one task per step, same rows, padded steps on the pad
+// token [G2] -- and every request of the batch completes when its last task retires.
+static int schedule_graph(Engine& e, std::vector<Task>& out) {
+  const int nb = static_cast<int>(e.buckets.size());
+  int pick = -1;
+  for (int d = 0; d < nb; ++d) {                        // cyclic scan after the last served
+    const int i = (e.last_bucket + 1 + d) % nb;
+    if (!e.buckets[i].empty()) {
+      pick = i;
+      break;
+    }
+  }
+  if (pick < 0) return 0;
+  std::deque<int>& q = e.buckets[pick];
+  const int ct = e.reqs[q.front()].cell0;
+  Cell& c = e.cells[ct];
+  const int n = std::min<int>({c.d.max_batch, static_cast<int>(q.size()),
+                               static_cast<int>(e.free_slots_heap.size())});
+  if (n == 0) return 0;
+  e.last_bucket = pick;
+  std::vector<int> rids(n);
+  for (int k = 0; k < n; ++k) {
+    rids[k] = q.front();
+    q.pop_front();
+    Request& r = e.reqs[rids[k]];
+    r.started = true;
+    r.slot = slot_alloc(e);                               // [G3]
+    r.t_first = e.now;
+  }
+  const int steps = (pick + 1) * e.cfg.bucket_width;     // the bucket's unrolled graph
+  for (int s = 0; s < steps; ++s) {
+    Task t;
+    t.ct = ct;
+    t.tick = e.now;
+    t.rows.reserve(n);
+    t.desc.reserve(n);
+    for (int ri : rids) {
+      const Request& r = e.reqs[ri];
+      t.rows.push_back({ri, s, r.slot});
+      RowDesc d{};
+      d.slot = r.slot;
+      d.a = s < r.n_nodes ? r.tokens[s] : 0;             // pad token past the request's end [G2]
+      int flags = 0;
+      if (s == 0) flags |= ROW_FIRST;
+      if (s & 1) flags |= ROW_PARITY;
+      if (s == r.n_nodes - 1) flags |= ROW_LAST;          // result row = the real last step
+      d.flags = flags | (ri << 8);
+      t.desc.push_back(d);
+    }
+    c.running_tasks += 1;
+    if (s == steps - 1) t.batch_reqs = rids;
+    out.push_back(std::move(t));
+  }
+  return steps;
+}
+
 // Schedule(worker), Alg. 1 lines 4-11. If the chosen type forms no task only because the
 // slot pool is exhausted, fall through to the next choice [S22].
 int schedule(Engine& e, std::vector<Task>& out) {
+  if (e.cfg.policy == BM_POLICY_GRAPH) return schedule_graph(e, out);
   const int worker = 0;
   const int nc = static_cast<int>(e.cells.size());
   uint64_t excluded = 0;
@@ -351,6 +419,26 @@ int schedule(Engine& e, std::vector<Task>& out) {
 void retire_task(Engine& e, Task& t) {
   Cell& c = e.cells[t.ct];
   c.running_tasks -= 1;
+  if (e.cfg.policy == BM_POLICY_GRAPH) {   // the graph returns every output at its end
+    for (int ri : t.batch_reqs) {
+      Request& r = e.reqs[ri];
+      r.done = true;
+      r.t_done = e.now;
+      bm_completion cp;
+      cp.req_id = r.id;
+      cp.user_tag = r.tag;
+      cp.t_arrival = r.t_arrival;
+      cp.t_first = r.t_first;
+      cp.t_done = r.t_done;
+      e.completions.push_back(cp);
+      slot_release(e, r.slot);
+      if (!e.cfg.keep_results) {
+        r.used = false;
+        e.n_live_reqs -= 1;
+      }
+    }
+    return;
+  }
   for (size_t i = 0; i < t.rows.size(); ++i) {
     const TaskRow& row = t.rows[i];
     Request& r = e.reqs[row.req];

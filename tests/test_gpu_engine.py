@@ -166,3 +166,31 @@ def test_persistent_large_batches_match_launch_path():
     for i in (0, 299, 599):
         hs, _ = cells.chain_lstm(w, trace[i].tokens)
         assert np.max(np.abs(res[1][i] - hs[0])) <= TOL[bm.PREC_BF16]
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+def test_graph_batching_policy_h1024(prec):
+    """N4: the padding + bucketing baseline (§7.1) on the same kernels -- task log and
+    completions bit-exact with its replay, and padding does not change any request's result
+    (the result row is the real last step; padded steps run on the pad token afterwards)."""
+    from oracle.scheduler import GraphBatchingReplay
+    trace = gen.chain_trace(40, 2048, seed=1001, rate=1.0)
+    e, cid, w = lstm_engine(1024, 1, 2048, prec, bmax=16, clock=bm.CLOCK_VIRTUAL, max_slots=256,
+                            max_requests=256, keep_results=1, schedule_when_outstanding_leq=1,
+                            policy=bm.POLICY_GRAPH, bucket_width=10)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    assert e.run() == len(trace)
+    rp = GraphBatchingReplay(16, max_slots=256, bucket_width=10, schedule_when_outstanding_leq=1)
+    rp.run([dict(arrival=q.arrival, length=q.length) for q in trace])
+    log = e.read_log()
+    assert len(log) == len(rp.tasks)
+    for a, t in zip(log, rp.tasks):
+        assert a["tick"] == t.tick and a["rows"] == [(r.rid, r.node, r.slot) for r in t.rows]
+    comp = e.poll()
+    assert [(c.req_id, c.t_done) for c in comp] == [(rid, float(tk)) for rid, tk in rp.completions]
+    for i, q in enumerate(trace):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, q.tokens)
+        assert np.max(np.abs(r["h"][0] - hs[0])) <= TOL[prec]
+        assert np.max(np.abs(r["c"][0] - cs[0])) <= TOL[prec]
