@@ -75,6 +75,8 @@ struct StepArgs {
   unsigned int dep_seq;       // this launch's sequence number (waits for dep_seq - 1)
   unsigned long long* tl;     // diagnostics (BM_TIMELINE): {~first CTA start, ~first past the
                               // PDL wait, last CTA end, CTAs} in %globaltimer ns, or null
+  int cbuf_off;               // set by the launcher: shared-memory offset (from the 1 KB-aligned
+                              // base) of the epilogue's prefetched c-state rows
 };
 
 // Persistent weight-stationary LSTM engine (lstm_persistent_sm100.cu).

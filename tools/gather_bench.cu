@@ -276,7 +276,7 @@ int main(int argc, char** argv) {
     for (int i = 0; i < 4; ++i) idx[i] = (i == 1) ? -1 : idx[i];  // a negative row: OOB -> zero fill?
     CK(cudaMemcpy(didx, idx.data(), idx.size() * 4, cudaMemcpyHostToDevice));
     const int nk = npad <= 64 ? 8 : (npad == 128 ? 8 : 6);
-    for (int mode : {3}) {
+    for (int mode : {0, 1, 2, 3, 5}) {
       gather_kernel<<<nsm, 256, 200 * 1024>>>(map, d, H, didx, npad, nk, mode, dout, share == 2, dimg, 20);
       CK(cudaGetLastError());
       CK(cudaDeviceSynchronize());
