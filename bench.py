@@ -165,6 +165,18 @@ def pct(a, q):
     return float(np.percentile(a, q)) if len(a) else float("nan")
 
 
+def load_traffic():
+    """roofline.traffic: per-launch DRAM bytes of the LSTM cell-step kernels from the newest
+    committed ncu summary (profiles/round*/traffic_*.json, tools/traffic_from_ncu.py)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "round*", "traffic_*.json")))
+    if not files:
+        return None
+    d = json.load(open(files[-1]))
+    d["file"] = os.path.relpath(files[-1], ROOT)
+    return d
+
+
 # ------------------------------------------------------------------------------ clocks
 class ClockSampler:
     """nvidia-smi clocks/throttle reasons sampled DURING the timed region."""
@@ -441,8 +453,12 @@ def main():
     achieved = st["timed_bytes"] / (t_kern / 1e3) / 1e9 if t_kern > 0 else 0.0
     tflops = st["timed_flops"] / (t_kern / 1e3) / 1e12 if t_kern > 0 else 0.0
     bf16_peak = peaks.get("bf16_tflops", 1590.0)
+    traffic = load_traffic() if wl == "lstm" and not a.persistent else None
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
-            "traffic": None, "kernel": kernel, "timing": timing, "launches": st["timed_launches"],
+            "traffic": traffic["dram_bytes_per_launch"] if traffic else None,
+            "traffic_unit": "bytes/launch (DRAM read+write, ncu, cold L2)",
+            "traffic_l2_to_sm": traffic["l2_to_sm_bytes_per_launch"] if traffic else None,
+            "traffic_source": traffic["file"] if traffic else None, "kernel": kernel, "timing": timing, "launches": st["timed_launches"],
             "avg_launch_us": t_kern * 1e3 / max(1, st["timed_launches"]),
             "avg_rows_per_task": st["rows"] / max(1, st["tasks"]), "tensor_tflops": tflops,
             "tensor_frac": tflops / bf16_peak,
