@@ -153,6 +153,18 @@ typedef struct {
   const int32_t* right;    /* TREE: [n] right child or -1                                 */
   double arrival;      /* WALL: seconds after bm_run start; VIRTUAL/DRY: tick             */
   uint64_t user_tag;   /* returned in bm_completion                                       */
+  /* SEQ2SEQ <eos>-terminated decoding (L715: "Decoding terminates when either
+   * the <eos> symbol is generated or when the maximum decoding length is reached"). eos_stop
+   * = 0 (zero-initialised default): decode exactly decode_len steps (the paper's protocol).
+   * eos_stop = 1: decode_len is the maximum length (<= 4095); the device marks the request
+   * finished when its argmax equals eos_id (0 <= eos_id < vocab); decoder steps the scheduler
+   * had already submitted (look-ahead, L379) are masked on the device and nothing further is
+   * scheduled. The scheduler learns of the <eos> at the retire of the task that emitted it.
+   * dry_eos_step: BM_CLOCK_DRY only (no device, scheduler tests): the decode step whose token
+   * the scheduler is told was <eos> (-1 = never).                                            */
+  int eos_stop;
+  int32_t eos_id;
+  int dry_eos_step;
 } bm_request;
 
 /* Admit a request (unfold, A1). All arrays are copied. The request becomes visible to the
@@ -193,7 +205,8 @@ bm_status bm_run(bm_engine* e, int* n_completed);
 typedef struct {
   float* h;          /* [layers][hidden] final hidden state (fp32), or NULL              */
   float* c;          /* [layers][hidden] final cell state, or NULL                       */
-  int32_t* tokens;   /* SEQ2SEQ: [decode_len] emitted tokens, or NULL                    */
+  int32_t* tokens;   /* SEQ2SEQ: [decode_len] emitted tokens, or NULL; with eos_stop the
+                        entries after the <eos> step are -1                                 */
   float* logits;     /* SEQ2SEQ with record_logits: [decode_len][vocab], or NULL          */
 } bm_result;
 
@@ -241,7 +254,9 @@ typedef struct {
 
 enum { BM_ROW_FIRST = 1,  /* h_prev = c_prev = 0 (first node of a request)                 */
        BM_ROW_LAST = 2,   /* write fp32 h, c of this row to result row (flags >> 8)        */
-       BM_ROW_PARITY = 4  /* LSTM: read h[parity], write h[1 - parity]                     */ };
+       BM_ROW_PARITY = 4, /* LSTM: read h[parity], write h[1 - parity]                     */
+       BM_ROW_EOS = 8     /* decoder row of an eos_stop request: b = step | (eos_id + 1) << 12;
+                             the row is a no-op once the slot's request emitted <eos>      */ };
 
 bm_status bm_cell_step(bm_engine* e, int cell_id, const bm_step_row* rows, int b, int async);
 

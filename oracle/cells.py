@@ -18,6 +18,7 @@ SURVEY.md §8c S1-S11):
   S6  Seq2Seq: L-layer encoder and L-layer decoder, one cell = one timestep of the stack.
   S7  decoder layer l starts from encoder layer l's final (h, c).
   S8/S9 greedy feed-previous for exactly T steps (L715); argmax ties -> lowest index.
+  N1  optional <eos> stop: the step emitting <eos> is the last, T is then the maximum (L715).
   S10 logits = W_out h_L + b_out.
   S11 TreeLSTM (binary N-ary form): leaf z = W_leaf x + b -> (i, o, u), c = i*u,
       h = o*tanh(c); internal z = U [h_L; h_R] + b -> (i, f_L, f_R, o, u),
@@ -93,12 +94,18 @@ def argmax_lowest(v: np.ndarray) -> int:
 
 
 def seq2seq(enc, dec, src_tokens: Sequence[int], decode_len: int,
-            forced_tokens: Optional[Sequence[int]] = None) -> Dict[str, object]:
-    """Encoder over the source, then greedy feed-previous decoding for exactly decode_len
-    steps (L713-L715). If forced_tokens is given (the GPU's emitted tokens, SURVEY §8c
-    "forced-token mode") the decoder feeds those instead of its own argmax, so that a
-    legitimate bf16 argmax flip does not desynchronise the comparison; the oracle's own
-    argmax is still returned for the validity check."""
+            forced_tokens: Optional[Sequence[int]] = None, eos_id: Optional[int] = None) -> Dict[str, object]:
+    """Encoder over the source, then greedy feed-previous decoding (L713-L715).
+
+    eos_id None: exactly decode_len steps (the paper's evaluation protocol, L715).
+    eos_id set: "Decoding terminates when either the <eos> symbol is generated or when the
+    maximum decoding length is reached" (L715, deployed systems) -- decode_len is then the
+    maximum length; the step that emits <eos> is the last one (its state is the result).
+
+    If forced_tokens is given (the GPU's emitted tokens, SURVEY §8c "forced-token mode") the
+    decoder feeds those instead of its own argmax -- and termination follows them too -- so
+    that a legitimate bf16 argmax flip does not desynchronise the comparison; the oracle's
+    own argmax is still returned for the validity check."""
     hs, cs = chain_lstm(enc, src_tokens)
     logits_all, own_tokens, fed = [], [], []
     prev = GO
@@ -110,6 +117,8 @@ def seq2seq(enc, dec, src_tokens: Sequence[int], decode_len: int,
         own_tokens.append(y)
         prev = int(forced_tokens[s]) if forced_tokens is not None else y
         fed.append(prev)
+        if eos_id is not None and prev == eos_id:
+            break
     return {"h": hs, "c": cs, "logits": np.array(logits_all), "tokens": own_tokens,
             "fed_tokens": fed}
 

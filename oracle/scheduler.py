@@ -88,6 +88,7 @@ class Req:
         self.leaves_left = 0
         self.enc_len = 0
         self.internal_sg: Optional[Subgraph] = None
+        self.eos_step: Optional[int] = None
 
 
 class SlotPool:
@@ -144,7 +145,10 @@ class Replay:
 
     # ------------------------------------------------------------ request processor (A1)
     def admit(self, kind: int, cells: Sequence[int], length: int = 0, decode_len: int = 0,
-              left: Optional[Sequence[int]] = None, right: Optional[Sequence[int]] = None) -> int:
+              left: Optional[Sequence[int]] = None, right: Optional[Sequence[int]] = None,
+              eos_step: Optional[int] = None) -> int:
+        """eos_step (SEQ2SEQ, §8f N1): the decode step whose emitted token is <eos> -- an input
+        here (the tokens are data, not scheduling); decode_len is then the maximum length."""
         rid = len(self.reqs)
         if kind == CHAIN:
             r = Req(rid, kind, length)
@@ -199,6 +203,7 @@ class Replay:
                 sg.ready = [sg.nodes[0]]
         else:
             raise ValueError(kind)
+        r.eos_step = eos_step if kind == SEQ2SEQ else None
         self.reqs.append(r)
         return rid
 
@@ -326,6 +331,8 @@ class Replay:
         for row in task.rows:
             r = self.reqs[row.rid]
             sg = r.node_sg[row.node]
+            if r.eos_step is not None and row.node - r.enc_len == r.eos_step:
+                self._truncate_decoder(r, sg)
             if sg not in seen:
                 seen.append(sg)
                 sg.inflight -= 1
@@ -340,6 +347,18 @@ class Replay:
                 self.completions.append((r.rid, self.now))
                 for s in sorted(set(r.slots.values())):
                     self.pool.release(s)
+
+    def _truncate_decoder(self, r: Req, sg: Subgraph):
+        """§8f N1, L715: "Decoding terminates when ... the <eos> symbol is generated". The
+        scheduler learns it when the task holding the <eos> step retires (the token is computed
+        on the device); decoder steps submitted after it (look-ahead, L379) still run -- masked
+        on the device -- and retire, nothing further is submitted, and the request completes
+        at the retire of its last submitted node."""
+        sg.nodes = sg.nodes[:sg.n_submitted]
+        sg.ready = []
+        if sg in sg.ct.queue:
+            sg.ct.queue.remove(sg)
+        r.n_nodes = r.enc_len + len(sg.nodes)
 
     def _subgraph_done(self, sg: Subgraph):
         r = sg.req
@@ -371,7 +390,8 @@ class Replay:
                 i = pending.pop(0)
                 q = requests[i]
                 rid_of[i] = self.admit(q["kind"], q["cells"], q.get("length", 0),
-                                       q.get("decode_len", 0), q.get("left"), q.get("right"))
+                                       q.get("decode_len", 0), q.get("left"), q.get("right"),
+                                       q.get("eos_step"))
             if len(self.inflight) <= self.k:
                 for task in self.schedule(0):
                     start = max(t, self.last_finish)

@@ -53,7 +53,8 @@ class Request(C.Structure):
     _fields_ = [("kind", C.c_int), ("cell0", C.c_int), ("cell1", C.c_int), ("n", C.c_int),
                 ("tokens", C.POINTER(C.c_int32)), ("decode_len", C.c_int),
                 ("left", C.POINTER(C.c_int32)), ("right", C.POINTER(C.c_int32)),
-                ("arrival", C.c_double), ("user_tag", C.c_uint64)]
+                ("arrival", C.c_double), ("user_tag", C.c_uint64),
+                ("eos_stop", C.c_int), ("eos_id", C.c_int32), ("dry_eos_step", C.c_int)]
 
 
 class Completion(C.Structure):
@@ -214,12 +215,16 @@ class Engine:
 
     # ---------------------------------------------------------------- requests
     def submit(self, kind: int, cell0: int, cell1: int, tokens, arrival: float = 0.0,
-               decode_len: int = 0, left=None, right=None, tag: int = 0) -> int:
+               decode_len: int = 0, left=None, right=None, tag: int = 0,
+               eos_id: Optional[int] = None, dry_eos_step: int = -1) -> int:
+        """eos_id (SEQ2SEQ): stop decoding at <eos> = eos_id, decode_len is then the maximum
+        length (bm_request.eos_stop); dry_eos_step: BM_CLOCK_DRY scheduler tests only."""
         t = _i32(tokens)
         l = _i32(left) if left is not None else None
         r = _i32(right) if right is not None else None
         q = Request(kind, cell0, cell1, len(t), _ip(t), decode_len, _ip(l), _ip(r),
-                    float(arrival), tag)
+                    float(arrival), tag, 1 if eos_id is not None else 0,
+                    eos_id if eos_id is not None else -1, dry_eos_step)
         rid = C.c_uint64()
         _ck(lib.bm_submit(self.h, C.byref(q), C.byref(rid)), "bm_submit")
         return rid.value

@@ -129,6 +129,12 @@ __global__ void __launch_bounds__(kThreads) cell_step_simt_kernel(const __grid_c
       cn = sigm(z[0]) * tanhf(z[4]) + sigm(z[1]) * cl + sigm(z[2]) * cr;
       hn = sigm(z[3]) * tanhf(cn);
     }
+    if constexpr (EPI == EPI_LSTM) {  // N1: rows of a request that emitted <eos> are no-ops
+      if (p.dead != nullptr) {
+        if ((r.flags & ROW_EOS) && p.dead[r.slot]) continue;
+        if (p.layer == 0 && (r.flags & ROW_FIRST) && u == 0) p.dead[r.slot] = 0;  // slot's new owner
+      }
+    }
     p.c_pool[r.slot * H + u] = cn;
     const int par_out = (EPI == EPI_LSTM) ? ((r.flags & ROW_PARITY) ? 0 : 1) : 0;
     hp[(par_out * NS + r.slot) * H + u] = hn;
@@ -191,7 +197,9 @@ __global__ void __launch_bounds__(kThreads) proj_simt_kernel(const __grid_consta
     float z = acc[c] + bias;
     if (p.logits != nullptr && col < p.b) {
       const RowDesc rd = p.rows[col];
-      p.logits[(static_cast<size_t>(rd.flags >> 8) * p.max_decode + rd.b) * p.V + v0 + r] = z;
+      const bool skip = (rd.flags & ROW_EOS) && p.dead != nullptr && p.dead[rd.slot];
+      const int step = (rd.flags & ROW_EOS) ? row_step(rd.b) : rd.b;
+      if (!skip) p.logits[(static_cast<size_t>(rd.flags >> 8) * p.max_decode + step) * p.V + v0 + r] = z;
     }
     int zi = v0 + r;
     for (int o = 16; o > 0; o >>= 1) {  // warp argmax, lowest index on ties
@@ -235,8 +243,16 @@ __global__ void __launch_bounds__(kThreads) proj_simt_kernel(const __grid_consta
       const RowDesc rd = p.rows[c];
       const unsigned long long key = atomicExch(p.amax + c, 0ull);
       const int y = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(key & 0xFFFFFFFFull));
+      const bool eos_row = (rd.flags & ROW_EOS) && p.dead != nullptr;
+      if (eos_row && p.dead[rd.slot]) continue;  // N1: masked step after the request's <eos>
+      const int step = (rd.flags & ROW_EOS) ? row_step(rd.b) : rd.b;
       p.tok[rd.slot] = y;
-      p.res_tok[static_cast<size_t>(rd.flags >> 8) * p.max_decode + rd.b] = y;
+      p.res_tok[static_cast<size_t>(rd.flags >> 8) * p.max_decode + step] = y;
+      if (eos_row && y == row_eos(rd.b)) {  // <eos> emitted: later steps of the request are no-ops
+        p.dead[rd.slot] = 1;
+        p.eos_host[rd.flags >> 8] = step + 1;
+        __threadfence_system();
+      }
     }
     if (tid == 0) *p.done_ctas = 0;
   }

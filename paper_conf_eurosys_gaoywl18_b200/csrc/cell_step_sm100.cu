@@ -461,8 +461,10 @@ __global__ void __launch_bounds__(kThreads, 2)
       float best = -INFINITY;
       int besti = 0;
       float* lg = nullptr;
-      if (p.logits != nullptr) {
-        lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + r.b) * p.V + v0;
+      const bool masked = (r.flags & ROW_EOS) && p.dead != nullptr && p.dead[r.slot];
+      if (p.logits != nullptr && !masked) {
+        const int step = (r.flags & ROW_EOS) ? row_step(r.b) : r.b;
+        lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + step) * p.V + v0;
       }
       for (int i = 0; i < 128; ++i) {
         const float z = P[c * pitch + i] + p.bias[v0 + i];
@@ -492,8 +494,16 @@ __global__ void __launch_bounds__(kThreads, 2)
         const RowDesc r = row_at(p, rr, c);
         const unsigned long long key = atomicExch(p.amax + c, 0ull);
         const int y = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(key & 0xFFFFFFFFull));
+        const bool eos_row = (r.flags & ROW_EOS) && p.dead != nullptr;
+        if (eos_row && p.dead[r.slot]) continue;  // N1: masked step after the request's <eos>
+        const int step = (r.flags & ROW_EOS) ? row_step(r.b) : r.b;
         p.tok[r.slot] = y;
-        p.res_tok[static_cast<size_t>(r.flags >> 8) * p.max_decode + r.b] = y;
+        p.res_tok[static_cast<size_t>(r.flags >> 8) * p.max_decode + step] = y;
+        if (eos_row && y == row_eos(r.b)) {  // <eos> emitted: later steps of the request are no-ops
+          p.dead[r.slot] = 1;
+          p.eos_host[r.flags >> 8] = step + 1;
+          __threadfence_system();
+        }
       }
       __threadfence();
       __syncthreads();
@@ -622,6 +632,12 @@ __global__ void __launch_bounds__(kThreads, 2)
               continue;
             }
             const RowDesc& rr_ = r[h];
+            if constexpr (EPI == EPI_LSTM) {  // N1: rows of a request that emitted <eos> are no-ops
+              if (p.dead != nullptr) {
+                if ((rr_.flags & ROW_EOS) && p.dead[rr_.slot]) continue;
+                if (p.layer == 0 && (rr_.flags & ROW_FIRST) && u == 0) p.dead[rr_.slot] = 0;
+              }
+            }
             p.c_pool[rr_.slot * H + u] = cn;
             const int par_out = (EPI == EPI_LSTM) ? ((rr_.flags & ROW_PARITY) ? 0 : 1) : 0;
             static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + rr_.slot) * H + u] = __float2bfloat16_rn(hn);
@@ -1108,6 +1124,10 @@ __global__ void __launch_bounds__(kThreads, 1)
           const float cn = sigm(z1) * cin[h] + sigm(z0) * tanh_f(z2);
           const float hn = sigm(z3) * tanh_f(cn);
           const RowDesc& rw = r[h];
+          if (p.dead != nullptr) {  // N1: rows of a request that emitted <eos> are no-ops
+            if ((rw.flags & ROW_EOS) && p.dead[rw.slot]) continue;
+            if (p.layer == 0 && (rw.flags & ROW_FIRST) && u == 0) p.dead[rw.slot] = 0;
+          }
           p.c_pool[rw.slot * H + u] = cn;
           const int par_out = (rw.flags & ROW_PARITY) ? 0 : 1;
           static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + rw.slot) * H + u] = __float2bfloat16_rn(hn);

@@ -96,6 +96,12 @@ struct Request {
   int slot = -1;            // chain / seq2seq
   int leaves_left = 0;
   int internal_sid = -1;
+  // <eos>-terminated decoding (§8f N1)
+  bool eos_stop = false;
+  int eos_id = -1;
+  int eos_step = -1;        // decode step of the <eos>, once the scheduler has learned it
+  int dry_eos_step = -1;    // BM_CLOCK_DRY: the step reported as <eos>
+  int decode_max = 0;       // decode_len as submitted (maximum length under eos_stop)
   bool used = false;
   bool done = false;
   bool started = false;     // slots taken
@@ -184,6 +190,9 @@ struct Engine {
   void* h_pool = nullptr;          // [layers][2][slots][H]
   float* c_pool = nullptr;         // [layers][slots][H]
   int* tok = nullptr;              // [slots]
+  int* dead = nullptr;             // [slots] device: request emitted <eos> (N1)
+  int* eos_host = nullptr;         // [max_requests] pinned, mapped: <eos> step + 1 (N1)
+  int* eos_dev = nullptr;          // device pointer of eos_host
   float* res_h = nullptr;          // [max_requests][layers][H]
   float* res_c = nullptr;
   int32_t* res_tok = nullptr;      // [max_requests][max_decode]

@@ -14,7 +14,10 @@ struct RowDesc {
   int32_t slot;   // output slot (LSTM: also the state read)
   int32_t flags;  // ROW_* | result_index << 8
 };
-enum { ROW_FIRST = 1, ROW_LAST = 2, ROW_PARITY = 4 };
+enum { ROW_FIRST = 1, ROW_LAST = 2, ROW_PARITY = 4, ROW_EOS = 8 };
+// ROW_EOS rows (decoder of an <eos>-terminated request, §8f N1): b = decode step | (eos + 1) << 12
+__host__ __device__ inline int row_step(int b) { return b & 0xFFF; }
+__host__ __device__ inline int row_eos(int b) { return (b >> 12) - 1; }
 
 // Epilogue kinds (template parameter of the kernels).
 enum { EPI_LSTM = 0, EPI_PROJ = 1, EPI_LEAF = 2, EPI_INTERNAL = 3 };
@@ -75,6 +78,9 @@ struct StepArgs {
   unsigned int dep_seq;       // this launch's sequence number (waits for dep_seq - 1)
   unsigned long long* tl;     // diagnostics (BM_TIMELINE): {~first CTA start, ~first past the
                               // PDL wait, last CTA end, CTAs} in %globaltimer ns, or null
+  int* dead;                  // [n_slots] 1 once the slot's request emitted <eos> (ROW_EOS rows
+                              // are then no-ops); cleared by the request's first encoder step
+  int* eos_host;              // host-mapped [max_requests]: decode step + 1 of the <eos>, or 0
   int cbuf_off;               // set by the launcher: shared-memory offset (from the 1 KB-aligned
                               // base) of the epilogue's prefetched c-state rows
 };

@@ -100,6 +100,8 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
   a.h_pool = e.h_layer(pl);
   a.c_pool = e.c_layer(pl);
   a.tok = e.tok;
+  a.dead = e.dead;
+  a.eos_host = e.eos_dev;
   a.W = proj ? c.W_out : c.W[layer];
   a.bias = proj ? c.b_out : c.bias[layer];
   a.W_rows = proj ? c.d.vocab : c.G * e.cfg.hidden;
@@ -472,6 +474,8 @@ static void free_device(Engine& e) {
   cudaFree(e.h_pool);
   cudaFree(e.c_pool);
   cudaFree(e.tok);
+  cudaFree(e.dead);
+  if (e.eos_host) cudaFreeHost(e.eos_host);
   cudaFree(e.res_h);
   cudaFree(e.res_c);
   cudaFree(e.res_tok);
@@ -541,6 +545,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
     const size_t el = E.elem();
     bool ok = cudaMalloc(&E.h_pool, L * 2 * S * H * el) == cudaSuccess &&
               dalloc(&E.c_pool, L * S * H) == cudaSuccess && dalloc(&E.tok, S) == cudaSuccess &&
+              dalloc(&E.dead, S) == cudaSuccess &&
               dalloc(&E.res_h, R * L * H) == cudaSuccess && dalloc(&E.res_c, R * L * H) == cudaSuccess &&
               dalloc(&E.res_tok, R * static_cast<size_t>(c.max_decode_len)) == cudaSuccess &&
               dalloc(&E.amax, 512) == cudaSuccess && dalloc(&E.done_ctas, 1) == cudaSuccess &&
@@ -558,6 +563,11 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
                       cudaHostAllocMapped) != cudaSuccess)
       return fail(BM_E_NOMEM);
     *E.signal_host = 0;
+    // <eos> reports (N1): written by the projection kernel, read at retire
+    if (cudaHostAlloc(reinterpret_cast<void**>(&E.eos_host), R * sizeof(int), cudaHostAllocMapped) != cudaSuccess ||
+        cudaHostGetDevicePointer(reinterpret_cast<void**>(&E.eos_dev), E.eos_host, 0) != cudaSuccess)
+      return fail(BM_E_NOMEM);
+    memset(E.eos_host, 0, R * sizeof(int));
     // ring-row publication flag (device) + the stream-write entry point (or a pinned value ring)
     if (dalloc(&E.rows_flag_dev, 1) != cudaSuccess ||
         cudaHostAlloc(reinterpret_cast<void**>(&E.rows_seq_host), 256 * sizeof(unsigned int),
@@ -576,6 +586,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
     if (cudaMemsetAsync(E.h_pool, 0, L * 2 * S * H * el, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.c_pool, 0, L * S * H * 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.tok, 0, S * 4, E.stream) != cudaSuccess ||
+        cudaMemsetAsync(E.dead, 0, S * 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.amax, 0, 512 * 8, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.done_ctas, 0, 4, E.stream) != cudaSuccess ||
         cudaMemsetAsync(E.sig_ctas, 0, 4, E.stream) != cudaSuccess ||
@@ -753,6 +764,8 @@ bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
       return BM_E_INVAL;
     if (q->decode_len < 1 || q->decode_len > e.cfg.max_decode_len) return BM_E_INVAL;
     if (e.cells[q->cell0].d.layers != e.cells[q->cell1].d.layers) return BM_E_INVAL;
+    if (q->eos_stop && (q->eos_id < 0 || q->eos_id >= e.cells[q->cell1].d.vocab || q->decode_len > 4095))
+      return BM_E_INVAL;
     vocab = e.cells[q->cell0].d.vocab;
   } else if (q->kind == BM_REQ_TREE) {
     if (!cell_ok(q->cell0, BM_CELL_TREE_LEAF, BM_CELL_TREE_LEAF) ||
@@ -781,6 +794,10 @@ bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
   r.cell1 = q->cell1;
   r.t_arrival = q->arrival;
   r.tokens.assign(q->tokens, q->tokens + q->n);
+  r.eos_stop = q->kind == BM_REQ_SEQ2SEQ && q->eos_stop != 0;
+  r.eos_id = r.eos_stop ? q->eos_id : -1;
+  r.dry_eos_step = r.eos_stop ? q->dry_eos_step : -1;
+  r.decode_max = q->kind == BM_REQ_SEQ2SEQ ? q->decode_len : 0;
   if (q->kind == BM_REQ_CHAIN) {
     r.n_nodes = q->n;
     r.enc_len = q->n;
@@ -1008,10 +1025,14 @@ bm_status bm_read_result(bm_engine* h, uint64_t req_id, bm_result* dst) {
   if (dst->h) CK(cudaMemcpyAsync(dst->h, e.res_h + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost, e.stream));
   if (dst->c) CK(cudaMemcpyAsync(dst->c, e.res_c + ri * L * H, L * H * 4, cudaMemcpyDeviceToHost, e.stream));
   if (r.kind == BM_REQ_SEQ2SEQ) {
-    const int T = r.n_nodes - r.enc_len;
-    if (dst->tokens)
+    // emitted tokens: up to and including the <eos> step under eos_stop (N1), else all steps
+    const int T = r.eos_step >= 0 ? r.eos_step + 1 : r.n_nodes - r.enc_len;
+    if (dst->tokens) {
       CK(cudaMemcpyAsync(dst->tokens, e.res_tok + static_cast<size_t>(ri) * e.cfg.max_decode_len, T * 4,
                          cudaMemcpyDeviceToHost, e.stream));
+      CK(cudaStreamSynchronize(e.stream));
+      for (int s = T; s < r.decode_max; ++s) dst->tokens[s] = -1;
+    }
     if (dst->logits && e.logits)
       CK(cudaMemcpyAsync(dst->logits, e.logits + static_cast<size_t>(ri) * e.cfg.max_decode_len * e.logits_vocab,
                          static_cast<size_t>(T) * e.logits_vocab * 4, cudaMemcpyDeviceToHost, e.stream));

@@ -113,6 +113,8 @@ bm_status admit_request(Engine& e, int ri) {
   r.slot = -1;
   r.t_first = -1;
   r.t_done = -1;
+  r.eos_step = -1;
+  if (e.eos_host != nullptr) e.eos_host[ri] = 0;  // no device write can be pending: entry free
   if (e.cfg.policy == BM_POLICY_GRAPH) {  // padding + bucketing: bucket (i*w, (i+1)*w] (L427)
     const size_t i = static_cast<size_t>((r.n_nodes - 1) / e.cfg.bucket_width);
     if (e.buckets.size() <= i) e.buckets.resize(i + 1);
@@ -259,6 +261,10 @@ RowDesc describe_row(const Request& r, int ri, int node, int slot) {
       const int s = step - r.enc_len;
       d.a = s == 0 ? 1 /* <go> */ : -1 /* feed previous: tok[slot] on device */;
       d.b = s;
+      if (r.eos_stop) {  // N1: any step may be the last -> every step writes the result row
+        flags |= ROW_EOS | ROW_LAST;
+        d.b = s | ((r.eos_id + 1) << 12);
+      }
     }
     if (step == r.n_nodes - 1) flags |= ROW_LAST;
   }
@@ -444,6 +450,20 @@ void retire_task(Engine& e, Task& t) {
     Request& r = e.reqs[row.req];
     const int sid = r.sid_of(row.node);
     Subgraph& g = r.sg(sid);
+    if (r.eos_stop && r.eos_step < 0 && sid == 1) {
+      // N1 (L715): did this row's decode step emit <eos>? Only the retire of the task holding
+      // that step acts on it (tasks retire in order), so the replay can follow the same rule.
+      const int s = row.node - r.enc_len;
+      const int rep = e.device() ? static_cast<volatile int*>(e.eos_host)[row.req] - 1 : r.dry_eos_step;
+      if (rep == s) {
+        r.eos_step = s;
+        // nothing more is submitted: the decoder ends with the nodes already in flight
+        if (g.queued) dequeue(e, row.req, 1);
+        g.ready.clear();
+        g.n_nodes = g.n_submitted;
+        r.n_nodes = r.enc_len + g.n_nodes;
+      }
+    }
     bool seen = false;  // rows of one subgraph are contiguous (see submit)
     if (i > 0 && t.rows[i - 1].req == row.req) {
       const TaskRow& o = t.rows[i - 1];

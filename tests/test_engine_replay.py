@@ -41,8 +41,10 @@ def _submit_all(e, reqs):
         if q["kind"] == CHAIN:
             e.submit(bm.REQ_CHAIN, q["cells"][0], 0, [3] * q["length"], q["arrival"])
         elif q["kind"] == SEQ2SEQ:
+            eos = q.get("eos_step")
             e.submit(bm.REQ_SEQ2SEQ, q["cells"][0], q["cells"][1], [3] * q["length"], q["arrival"],
-                     decode_len=q["decode_len"])
+                     decode_len=q["decode_len"], eos_id=5 if "eos_step" in q else None,
+                     dry_eos_step=-1 if eos is None else eos)
         else:
             n = len(q["left"])
             e.submit(bm.REQ_TREE, q["cells"][0], q["cells"][1], [3] * n, q["arrival"],
@@ -100,7 +102,7 @@ def test_complete_tree_replay():
     _compare(e, Replay([(64, 0), (64, 1)], max_slots=256).run(reqs))
 
 
-def _random_reqs(seed, n, kinds):
+def _random_reqs(seed, n, kinds, eos=False):
     rng = np.random.default_rng(seed)
     out = []
     t = 0.0
@@ -110,8 +112,12 @@ def _random_reqs(seed, n, kinds):
         if kind == CHAIN:
             out.append({"kind": CHAIN, "cells": [0], "arrival": t, "length": int(rng.integers(1, 9))})
         elif kind == SEQ2SEQ:
-            out.append({"kind": SEQ2SEQ, "cells": [1, 2], "arrival": t,
-                        "length": int(rng.integers(1, 6)), "decode_len": int(rng.integers(1, 6))})
+            q = {"kind": SEQ2SEQ, "cells": [1, 2], "arrival": t,
+                 "length": int(rng.integers(1, 6)), "decode_len": int(rng.integers(1, 9))}
+            if eos:  # <eos> at a random step, or never (N1)
+                st_ = int(rng.integers(0, q["decode_len"] + 2))
+                q["eos_step"] = st_ if st_ < q["decode_len"] else None
+            out.append(q)
         else:
             left, right = gen._random_bracketing(int(rng.integers(1, 9)), rng)
             out.append({"kind": TREE, "cells": [3, 4], "arrival": t, "left": left, "right": right})
@@ -152,3 +158,34 @@ def test_schedule_step_api_matches_run():
         assert n < 1000
     rp = Replay([(4, 0)], max_slots=16).run(reqs)
     _compare(e, rp)
+
+
+@settings(max_examples=150, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 100_000), n=st.integers(1, 16),
+       bmax=st.lists(st.integers(1, 6), min_size=5, max_size=5),
+       prio=st.permutations([0, 1, 2, 3, 4]), max_tasks=st.integers(1, 5),
+       k=st.integers(0, 3), slots=st.integers(4, 40),
+       kinds=st.sampled_from([[SEQ2SEQ], [CHAIN, SEQ2SEQ, TREE]]))
+def test_random_eos_traces_bit_exact(seed, n, bmax, prio, max_tasks, k, slots, kinds):
+    """§8f N1: <eos>-terminated decoding. The engine learns each request's <eos> at the retire
+    of the task that emitted it (BM_CLOCK_DRY: reported via dry_eos_step) and stops scheduling
+    its decoder; the replay follows the same rule independently. Logs and completions equal."""
+    reqs = _random_reqs(seed, n, kinds, eos=True)
+    need = max((len(q["left"]) if q["kind"] == TREE else 1) for q in reqs)
+    slots = max(slots, need)
+    kinds_c = [bm.CELL_LSTM, bm.CELL_LSTM, bm.CELL_LSTM_PROJ, bm.CELL_TREE_LEAF, bm.CELL_TREE_INTERNAL]
+    e, _ = _engine(list(zip(kinds_c, bmax, prio)), max_slots=slots, max_requests=64,
+                   max_tasks_to_submit=max_tasks, schedule_when_outstanding_leq=k)
+    _submit_all(e, reqs)
+    e.run()
+    rp = Replay(list(zip(bmax, prio)), max_slots=slots, max_tasks_to_submit=max_tasks,
+                schedule_when_outstanding_leq=k).run(reqs)
+    _compare(e, rp)
+
+
+def test_eos_request_rejected_when_invalid():
+    e, ids = _engine([(bm.CELL_LSTM, 4, 0), (bm.CELL_LSTM_PROJ, 4, 1)], max_slots=16, max_requests=16)
+    with pytest.raises(RuntimeError):
+        e.submit(bm.REQ_SEQ2SEQ, ids[0], ids[1], [3, 4], 0, decode_len=4, eos_id=128)  # >= vocab
+    with pytest.raises(RuntimeError):
+        e.submit(bm.REQ_SEQ2SEQ, ids[0], ids[1], [3, 4], 0, decode_len=4, eos_id=-2)

@@ -105,6 +105,71 @@ def test_seq2seq_forced_tokens(prec, h, V, n):
             assert np.max(np.abs(r["c"][l] - o["c"][l])) <= tol
 
 
+def _s2s_trace(V, n, seed):
+    rng = np.random.default_rng(seed)
+    trace = []
+    for i in range(n):
+        S = int(rng.integers(1, 12))
+        T = int(rng.integers(4, 14))
+        trace.append((rng.integers(3, V, size=S).astype(np.int32), T, float(rng.integers(0, 6))))
+    trace.sort(key=lambda x: x[2])
+    return trace
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+@pytest.mark.parametrize("h,V,n", [(64, 256, 12), (1024, 32768, 6)])
+def test_seq2seq_eos_terminated(prec, h, V, n):
+    """§8f N1 (L715): decoding stops at <eos> or at the maximum length. The <eos> symbol is the
+    token request 0 emits at some step j >= 1 in a fixed-length run, so at least one request
+    terminates early (with V = 256 others do too). Checked: tokens after each request's <eos>
+    are -1; the task log and completions are bit-exact with the replay given the <eos> steps
+    the device produced (the replay learns each at the retire of its task, like the engine);
+    the oracle in forced-token mode, stopping at the same <eos>, matches the emitted steps'
+    logits and the final h/c of every layer (the state of the <eos> step: later, speculatively
+    submitted steps were masked on the device)."""
+    L = 4
+    trace = _s2s_trace(V, n, h + 7)
+    kw = dict(bmax=(512, 256), clock=bm.CLOCK_VIRTUAL, max_slots=64, max_requests=64, keep_results=1,
+              record_logits=1, max_decode_len=40)
+    e, (ce, cd), (enc, dec) = seq2seq_engine(h, L, V, prec, **kw)
+    for toks, T, t in trace:
+        e.submit(bm.REQ_SEQ2SEQ, ce, cd, toks, t, decode_len=T)
+    e.run()
+    y0 = e.read_result(0, L, decode_len=trace[0][1])["tokens"]
+    j = next(i for i in range(1, len(y0)) if y0[i] not in y0[:i]) if len(set(y0)) > 1 else 0
+    eos = int(y0[j])
+    e.close()
+
+    e, (ce, cd), (enc, dec) = seq2seq_engine(h, L, V, prec, **kw)
+    for toks, T, t in trace:
+        e.submit(bm.REQ_SEQ2SEQ, ce, cd, toks, t, decode_len=T, eos_id=eos)
+    e.run()
+    tol = TOL[prec]
+    steps = []
+    for i, (toks, T, _) in enumerate(trace):
+        r = e.read_result(i, L, decode_len=T, vocab=V)
+        y = [int(v) for v in r["tokens"]]
+        m = y.index(-1) if -1 in y else T
+        assert all(v == -1 for v in y[m:])
+        assert all(v >= 0 for v in y[:m])
+        if m < T:
+            assert y[m - 1] == eos and eos not in y[:m - 1]
+        steps.append(m - 1 if m < T or (m == T and y[T - 1] == eos) else None)
+        o = cells.seq2seq(enc, dec, toks, T, forced_tokens=y[:m], eos_id=eos)
+        assert len(o["tokens"]) == m
+        for s in range(m):
+            assert o["logits"][s][y[s]] >= o["logits"][s].max() - 2 * tol
+        assert np.max(np.abs(r["logits"][:m] - o["logits"])) <= tol
+        for l in range(L):
+            assert np.max(np.abs(r["h"][l] - o["h"][l])) <= tol
+            assert np.max(np.abs(r["c"][l] - o["c"][l])) <= tol
+    assert steps[0] == j
+    reqs = [{"kind": SEQ2SEQ, "cells": [0, 1], "arrival": t, "length": len(toks), "decode_len": T,
+             "eos_step": steps[i]} for i, (toks, T, t) in enumerate(trace)]
+    _check_log(e, Replay([(512, 0), (256, 1)], max_slots=64).run(reqs))
+    e.close()
+
+
 @pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
 def test_treebank_trees_h1024(prec):
     """configs[3] shape: TreeBank-like binary trees + the identical complete 16-leaf tree,

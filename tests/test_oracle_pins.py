@@ -264,3 +264,36 @@ def test_p3_single_leaf_tree_is_leaf_cell():
     h2, c2 = cells.tree_leaf(w.W_leaf, w.b_leaf, w.E[9])
     np.testing.assert_array_equal(h, h2)
     np.testing.assert_array_equal(c, c2)
+
+
+# ---------------------------------------------------------------- §8f N1: <eos> termination
+def test_n1_seq2seq_eos_is_the_fixed_length_prefix():
+    """L715: "Decoding terminates when either the <eos> symbol is generated or when the
+    maximum decoding length is reached". With <eos> = v, the decode is the fixed-length decode
+    (pinned by P2) cut right after the first step that emits v: same tokens, same logits, same
+    final states as decoding exactly that many steps; a symbol never emitted changes nothing."""
+    from oracle import cells
+    enc = gen.lstm_stack_weights(32, 2, 16, seed=3, bf16=False, scale=4.0)
+    dec = gen.lstm_stack_weights(32, 2, 16, seed=103, projection=True, bf16=False, scale=4.0)
+    src = [3, 5, 7, 4]
+    T = 12
+    full = cells.seq2seq(enc, dec, src, T)
+    y = full["tokens"]
+    assert len(set(y)) >= 4  # several distinct symbols: several cut points
+    for v in sorted(set(y)):
+        e = y.index(v)
+        cut = cells.seq2seq(enc, dec, src, T, eos_id=v)
+        ref = cells.seq2seq(enc, dec, src, e + 1)
+        assert cut["tokens"] == y[:e + 1] and cut["tokens"][-1] == v
+        assert np.array_equal(cut["logits"], ref["logits"])
+        for l in range(2):
+            assert np.array_equal(cut["h"][l], ref["h"][l]) and np.array_equal(cut["c"][l], ref["c"][l])
+    never = [v for v in range(16) if v not in y]
+    if never:
+        out = cells.seq2seq(enc, dec, src, T, eos_id=never[0])
+        assert out["tokens"] == y and np.array_equal(out["h"][1], full["h"][1])
+    # forced-token mode terminates on the forced (device) tokens
+    forced = list(y)
+    forced[1] = 13
+    out = cells.seq2seq(enc, dec, src, T, forced_tokens=forced, eos_id=13)
+    assert len(out["tokens"]) == 2

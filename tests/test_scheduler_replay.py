@@ -209,3 +209,61 @@ def test_p7_fixed_length_throughput_bound():
     rp = _run_chain(trace, 64, 1)
     span = max(r.complete_tick for r in rp.reqs)
     assert len(trace) / span <= 64 / 24 + 1e-9
+
+
+# ---------------------------------------------------------------- §8f N1: <eos>-terminated decode
+def _s2s(length, T, eos_step, arrival=0.0):
+    return {"kind": SEQ2SEQ, "cells": [0, 1], "arrival": arrival, "length": length, "decode_len": T,
+            "eos_step": eos_step}
+
+
+@pytest.mark.parametrize("eos_step,n_tasks,complete", [(1, 7, 7.0), (4, 7, 7.0), (None, 8, 8.0), (0, 7, 7.0)])
+def test_n1_eos_hand_computed(eos_step, n_tasks, complete):
+    """One request, 2 encoder steps, at most 6 decoder steps, bmax 4, MaxTasks 5, idle-only
+    Schedule (k = 0), one tick per task. Tick 0: encoder tasks [e0] [e1] (successor ready at
+    submit, L381); tick 2: the encoder completes -> the decoder subgraph is released (L331) and
+    one Schedule call submits d0..d4 (MaxTasksToSubmit = 5, L379), finishing at ticks 3..7.
+    The <eos> is learned at the retire of its task (d1: tick 4; d4: tick 7); d0..d4 are already
+    in flight, so with <eos> at any step <= 4 nothing more is submitted and the request
+    completes at tick 7 (7 tasks). Without <eos> d5 runs at tick 7 -> completion at 8 (L715)."""
+    rp = Replay([(4, 0), (4, 1)]).run([_s2s(2, 6, eos_step)])
+    assert len(rp.tasks) == n_tasks
+    assert rp.completions == [(0, complete)]
+    assert [t.rows[0].node for t in rp.tasks] == list(range(n_tasks))
+
+
+@settings(max_examples=200, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 100_000), n=st.integers(1, 12), bmax=st.integers(1, 6),
+       max_tasks=st.integers(1, 5), k=st.integers(0, 3))
+def test_n1_eos_invariants(seed, n, bmax, max_tasks, k):
+    """For every request with <eos> at decode step e: the decoder ran steps 0..m-1 with
+    e < m <= T (nothing is skipped, the <eos> step ran, speculative steps are bounded by T); no
+    decoder step was submitted after the retire of the task that emitted <eos> (the scheduler
+    stops as soon as it learns of it); the request completes at the retire of its last
+    submitted node; requests without <eos> run all T steps."""
+    rng = np.random.default_rng(seed)
+    reqs, t = [], 0.0
+    for _ in range(n):
+        t += float(rng.integers(0, 3))
+        T = int(rng.integers(1, 9))
+        e = int(rng.integers(0, T + 2))
+        reqs.append(_s2s(int(rng.integers(1, 5)), T, e if e < T else None, t))
+    rp = Replay([(bmax, 0), (bmax, 1)], max_tasks_to_submit=max_tasks,
+                schedule_when_outstanding_leq=k).run(reqs)
+    done = dict(rp.completions)
+    for rid, q in enumerate(reqs):
+        L = q["length"]
+        dec = [(task, row.node - L) for task in rp.tasks for row in task.rows
+               if row.rid == rid and row.node >= L]
+        steps = sorted(s for _, s in dec)
+        m = len(steps)
+        assert steps == list(range(m))
+        last_finish = max(task.finish for task in rp.tasks for row in task.rows if row.rid == rid)
+        assert done[rid] == last_finish
+        if q["eos_step"] is None:
+            assert m == q["decode_len"]
+        else:
+            e = q["eos_step"]
+            assert e < m <= q["decode_len"]
+            t_eos = next(task.finish for task, s in dec if s == e)
+            assert all(task.tick < t_eos for task, _ in dec)
