@@ -426,16 +426,25 @@ def main():
     barrier()
     t0 = time.perf_counter()
     rows0 = e2.stats()["rows"]
+    ph = np.zeros(4)
     for _ in range(a.steps):
+        tp = [time.perf_counter()]
         fid = e2.submit_many(prep2)
+        tp.append(time.perf_counter())
         e2.run()
+        tp.append(time.perf_counter())
         e2.poll(n_req + 16)
+        tp.append(time.perf_counter())
         e2.read_results_many(fid, n_req, h=hbuf, release=True)
+        tp.append(time.perf_counter())
+        ph += np.diff(tp)
     e2e_s = allmax(time.perf_counter() - t0)
     rows_e2e = (e2.stats()["rows"] - rows0) / a.steps
     e2e = {"value": total / e2e_s, "unit": "requests/sec",
            "h2d_bytes_per_step": int(rows_e2e * 16),
-           "d2h_bytes_per_step": int(n_req * L * H * 4)}
+           "d2h_bytes_per_step": int(n_req * L * H * 4),
+           "host_ms_per_step": dict(zip(("submit", "run", "poll", "read_results"),
+                                        (float(x) for x in ph * 1e3 / a.steps)))}
     # ---- roofline of the dominant kernel (the LSTM / tree cell step), live CUDA events
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
