@@ -155,9 +155,9 @@ def run_trace(e, prepared, n):
     t0 = time.perf_counter()
     done = e.run()
     t1 = time.perf_counter()
-    comp = e.poll(n + 16)
+    comp = e.poll_array(n + 16)
     assert done == n and len(comp) == n, (done, len(comp), n)
-    lat = np.array([c.t_done - c.t_arrival for c in comp])
+    lat = comp["t_done"] - comp["t_arrival"]
     return t1 - t0, lat
 
 
@@ -401,8 +401,8 @@ def main():
             ev1.synchronize()
             assert done == n_req
             dev_ms += ev0.elapsed_time(ev1)
-            comp = e.poll(n_req + 16)
-            lats.append(np.array([c.t_done - c.t_arrival for c in comp]))
+            comp = e.poll_array(n_req + 16)
+            lats.append(comp["t_done"] - comp["t_arrival"])
     barrier()
     st = e.stats()
     lat = shard.gather_samples(np.concatenate(lats), dist, device=torch.device("cuda", local))
@@ -421,7 +421,7 @@ def main():
     for _ in range(max(1, a.warmup)):
         fid = e2.submit_many(prep2)
         e2.run()
-        e2.poll(n_req + 16)
+        e2.poll_array(n_req + 16)
         e2.read_results_many(fid, n_req, h=hbuf, release=True)
     barrier()
     t0 = time.perf_counter()
@@ -433,7 +433,7 @@ def main():
         tp.append(time.perf_counter())
         e2.run()
         tp.append(time.perf_counter())
-        e2.poll(n_req + 16)
+        e2.poll_array(n_req + 16)
         tp.append(time.perf_counter())
         e2.read_results_many(fid, n_req, h=hbuf, release=True)
         tp.append(time.perf_counter())

@@ -86,3 +86,14 @@ def test_malformed_trees_rejected():
         with pytest.raises(bm.BMError):
             e.submit(bm.REQ_TREE, leaf, intern, [3, 3, 3], left=left, right=right)
     e.submit(bm.REQ_TREE, leaf, intern, [3, 4, 0], left=[-1, -1, 1], right=[-1, -1, 0])
+
+
+def test_poll_array_layout_matches_bm_completion():
+    """bm.Engine.poll_array views bm_completion records as a numpy structured array: the dtype
+    must mirror the C struct (field order, offsets, size)."""
+    import ctypes as C
+    from paper_conf_eurosys_gaoywl18_b200 import bm
+    dt = bm.Engine._COMP_DT
+    assert dt.itemsize == C.sizeof(bm.Completion)
+    for name, _ in bm.Completion._fields_:
+        assert dt.fields[name][1] == getattr(bm.Completion, name).offset
