@@ -72,9 +72,9 @@ __host__ __device__ __forceinline__ int x_stages_for(int npad, int xring) {
 // wblk = one K block of the CTA's weight tile (tile rows x 128 B: 16 KB LSTM / projection,
 // 12 KB leaf, 10 KB internal)
 // xkb = K blocks per activation stage (one hand-off per stage)
-__host__ __device__ __forceinline__ int region_bytes(int npad, int wcb, int xring, int wblk, int xkb) {
+__host__ __device__ __forceinline__ int region_bytes(int pcols, int wcb, int xring, int wblk, int xkb, int npad) {
   const int a = kWRing * wcb * wblk + x_stages_for(npad * xkb, xring) * npad * xkb * 128;
-  const int b = 129 * npad * 4 + 4 * 128 * 4;
+  const int b = 129 * pcols * 4 + 4 * 128 * 4;  // partial / logits tile of pcols columns
   return a > b ? a : b;
 }
 
@@ -206,6 +206,38 @@ __device__ __forceinline__ const __nv_bfloat16* seg_src(const StepArgs& p, const
   } else {  // EPI_PROJ: h of the top layer, written at parity 1-par by this step
     const int par = (r.flags & ROW_PARITY) ? 1 : 0;
     return hp + ((1 - par) * S + r.slot) * H;
+  }
+}
+
+
+// Epilogue c-state prefetch (A9 inputs): the c rows this CTA's epilogue will read (LSTM: c of
+// the row's slot, zero for a first step; internal: c_L and c_R of the children), U units per
+// row, copied into shared memory by the producers with the first activation stage, so the
+// reduction loop does not wait on global loads. Layout: column cl (relative to c_lo) holds
+// nseg x U floats. The copies are covered by the stage's cp.async arrive (and a wait_all
+// before the epilogue).
+template <int EPI>
+__device__ __forceinline__ void prefetch_c(const StepArgs& p, const RowDesc* rtab, int c_lo, int my_cols,
+                                           int unit0, uint32_t cbuf, int t, int nthr) {
+  if constexpr (EPI == EPI_LSTM || EPI == EPI_INTERNAL) {
+    constexpr int nseg = EPI == EPI_INTERNAL ? 2 : 1;
+    const int cpc = nseg * p.U / 4;  // 16-byte chunks per column
+    const int cps = p.U / 4;         // chunks per segment
+    const size_t H = p.H;
+    for (int q = t; q < my_cols * cpc; q += nthr) {
+      const int cl = q / cpc, ch = q % cpc;
+      const RowDesc r = rtab[c_lo + cl];
+      const int seg = ch / cps;
+      const float* src;
+      bool zero = false;
+      if constexpr (EPI == EPI_LSTM) {
+        src = p.c_pool + static_cast<size_t>(r.slot) * H + unit0 + ch * 4;
+        zero = (r.flags & ROW_FIRST) != 0;
+      } else {
+        src = p.c_pool + static_cast<size_t>(seg ? r.b : r.a) * H + unit0 + (ch % cps) * 4;
+      }
+      cp_async_16(cbuf + q * 16, zero ? static_cast<const void*>(p.c_pool) : src, zero ? 0u : 16u);
+    }
   }
 }
 
@@ -359,6 +391,12 @@ __global__ void __launch_bounds__(kThreads, 2)
           }
         }
       }
+      if (st == 0 && EPI != EPI_PROJ && p.pchunk == 0) {
+        const int cper_ = (ncols + p.S - 1) / p.S;
+        const int clo_ = static_cast<int>(rank) * cper_;
+        prefetch_c<EPI>(p, rtab, clo_, max(0, min(ncols, clo_ + cper_) - clo_), blockIdx.y * U,
+                        smem_u32(base + p.cbuf_off), tid, kProducerThreads);
+      }
       cp_async_arrive_noinc(full0 + 8 * s);
       if (tid == 0 && st == 0) phase_mark(p, 10);
     }
@@ -433,6 +471,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   }
   if (warp < 8) {
     mbar_wait_warp(done_bar, 0);
+    asm volatile("cp.async.wait_all;" ::: "memory");  // own c-prefetch copies (already landed)
     tc_fence_after();
     if (tid == 0) phase_mark(p, 2);
   }
@@ -527,36 +566,43 @@ __global__ void __launch_bounds__(kThreads, 2)
     // (deterministic, independent of the batch's other rows). Posted scalar DSMEM stores
     // measured ~3x slower than these loads on B200.
     const int S = p.S;
-    const int cper = (ncols + S - 1) / S;
+    // exchange chunks (p.pchunk columns at a time; 0 = the whole tile): a chunk bounds the
+    // partial tile's shared memory so two CTAs fit on an SM (BM_PCHUNK experiments)
+    const bool chunked = p.pchunk > 0;  // launch-wide (the launcher then allocates no c prefetch)
+    const int CW = chunked ? min(p.pchunk, npad) : npad;
     float* P = reinterpret_cast<float*>(smem);
     constexpr int pitch = 128;
     // P row of tile row n = u * G + g: gates padded to Gp = 4 (G <= 4) or 8 (G = 5) floats per
     // unit, so a unit's gate values are one (or two) aligned 16-byte vector(s) for the reduction
     constexpr int Gp = (EPI == EPI_INTERNAL) ? 8 : 4;
     const int prow = (trow / G) * Gp + trow % G;
+    uint32_t peer[kMaxS];
+#pragma unroll
+    for (int s = 0; s < kMaxS; ++s) peer[s] = mapa(smem_u32(P), s < S ? s : 0);
+    const int unit0 = blockIdx.y * U;
+    const int prow0 = blockIdx.y * tile_rows;
+    const size_t H = p.H;
+    const size_t NS = p.n_slots;
+    for (int cc0 = 0; cc0 < npad; cc0 += CW) {
+    const int ccols = max(0, min(CW, ncols - cc0));
+    if (cc0 > 0) cluster_sync();  // peers are done reading the previous chunk's partials
     if (warp < 8) {
-      for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
+      for (int c0 = cc0 + (warp >> 2) * 32; c0 < cc0 + CW && c0 < npad; c0 += 64) {
         float v[32];
         tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
         if (trow < tile_rows) {
 #pragma unroll
           for (int i = 0; i < 32; ++i)
-            if (c0 + i < npad) P[(c0 + i) * pitch + prow] = v[i];
+            if (c0 + i < npad) P[(c0 - cc0 + i) * pitch + prow] = v[i];
         }
       }
     }
     tc_fence_before();
-    cluster_sync();  // A: every CTA's partial tile is in its smem
-    if (tid == 0) phase_mark(p, 3);
-    uint32_t peer[kMaxS];
-#pragma unroll
-    for (int s = 0; s < kMaxS; ++s) peer[s] = mapa(smem_u32(P), s < S ? s : 0);
-    const int c_lo = static_cast<int>(rank) * cper;
-    const int my_cols = max(0, min(ncols, c_lo + cper) - c_lo);
-    const int unit0 = blockIdx.y * U;
-    const int prow0 = blockIdx.y * tile_rows;
-    const size_t H = p.H;
-    const size_t NS = p.n_slots;
+    cluster_sync();  // A: every CTA's partial tile (chunk) is in its smem
+    if (tid == 0 && cc0 == 0) phase_mark(p, 3);
+    const int cper = (ccols + S - 1) / S;
+    const int c_lo = static_cast<int>(rank) * cper;   // relative to the chunk
+    const int my_cols = max(0, min(ccols, c_lo + cper) - c_lo);
     {
       // every warp takes part; each thread owns unit j of columns cl0, cl0 + step, ... and
       // handles two columns per iteration with all their loads issued up front (ILP: the
@@ -568,6 +614,7 @@ __global__ void __launch_bounds__(kThreads, 2)
 #pragma unroll
       for (int g = 0; g < 5; ++g) bias[g] = g < G ? p.bias[prow0 + j * G + g] : 0.f;
       const bool no_dsmem = (p.experiment & 32) != 0;  // diagnostics: own partial only
+      const float* cbuf = reinterpret_cast<const float*>(base + p.cbuf_off);
       for (int cl = tid / U; cl < my_cols; cl += 2 * ew) {
         if (tid == 0 && cl / (2 * ew) < 16) phase_mark(p, 32 + cl / (2 * ew));
         const int nit = (cl + ew < my_cols) ? 2 : 1;
@@ -585,15 +632,21 @@ __global__ void __launch_bounds__(kThreads, 2)
                 v[h][s] = ld_cluster_v4(a);
                 if (G == 5) w[h][s] = ld_cluster_v4(a + 16);
               }
-            r[h] = (p.experiment & 16) ? RowDesc{0, 0, (c_lo + cl + h * ew) & 1023, 0} : rtab[c_lo + cl + h * ew];
+            r[h] = (p.experiment & 16) ? RowDesc{0, 0, (c_lo + cl + h * ew) & 1023, 0}
+                                       : rtab[cc0 + c_lo + cl + h * ew];
             cin[h][0] = cin[h][1] = 0.f;
-            if (!(p.experiment & 16)) {
+            if (chunked) {  // no prefetch in chunked mode: c straight from the pool
               if constexpr (EPI == EPI_LSTM) {
                 if (!(r[h].flags & ROW_FIRST)) cin[h][0] = p.c_pool[r[h].slot * H + u];
               } else if constexpr (EPI == EPI_INTERNAL) {
                 cin[h][0] = p.c_pool[static_cast<size_t>(r[h].a) * H + u];
                 cin[h][1] = p.c_pool[static_cast<size_t>(r[h].b) * H + u];
               }
+            } else if constexpr (EPI == EPI_LSTM) {
+              cin[h][0] = cbuf[(cl + h * ew) * U + j];
+            } else if constexpr (EPI == EPI_INTERNAL) {
+              cin[h][0] = cbuf[(cl + h * ew) * 2 * U + j];
+              cin[h][1] = cbuf[(cl + h * ew) * 2 * U + U + j];
             }
           }
         }
@@ -650,6 +703,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         }
       }
     }
+    }  // chunk loop
     if (tid == 0) phase_mark(p, 4);
     cluster_sync();  // B: peers may read this CTA's partials until here
     if (tid == 0) phase_mark(p, 5);
@@ -727,9 +781,16 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
     a.xkb = 1;
   }
   const int wblk = (EPI == EPI_PROJ ? 128 : gates_of(EPI) * a.U) * 128;
-  const size_t smem = 1024 + kTailBytes + region_bytes(npad, a.wcb, a.xring, wblk, a.xkb);
-  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int S = EPI == EPI_PROJ ? 1 : a.S;
+  // epilogue c-state prefetch: ceil(cols / S) columns x 128 B (LSTM 32 units, internal 2 x 16)
+  static const int env_pchunk = getenv("BM_PCHUNK") ? atoi(getenv("BM_PCHUNK")) : 0;
+  a.pchunk = (EPI != EPI_PROJ && env_pchunk > 0 && env_pchunk % 64 == 0 && env_pchunk < npad) ? env_pchunk : 0;
+  const int cbuf_bytes = (EPI == EPI_LSTM || EPI == EPI_INTERNAL) && a.pchunk == 0
+                             ? (((cols + S - 1) / S) * (EPI == EPI_INTERNAL ? 2 : 1) * a.U * 4 + 1023) & ~1023
+                             : 0;
+  a.cbuf_off = kTailBytes + region_bytes(a.pchunk > 0 ? a.pchunk : npad, a.wcb, a.xring, wblk, a.xkb, npad);
+  const size_t smem = 1024 + a.cbuf_off + cbuf_bytes;
+  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(S, tiles, (a.b + kMaxCols - 1) / kMaxCols);
@@ -958,6 +1019,12 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       }
+      if (st == 0) {
+        const int cper_ = (ncols + p.S - 1) / p.S;
+        const int clo_ = ks * cper_;
+        prefetch_c<EPI_LSTM>(p, rtab, clo_, max(0, min(ncols, clo_ + cper_) - clo_), tile * U,
+                             smem_u32(base + p.cbuf_off), tid, kProducerThreads);
+      }
       cp_async_arrive_noinc(full0 + 8 * s);
       if (tid == 0 && st == 0) phase_mark(p, 10);
     }
@@ -1059,6 +1126,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   // ================================================================ epilogue (A9)
   wait_bounded_warp(done_bar, 0);
+  if (warp < 8) asm volatile("cp.async.wait_all;" ::: "memory");  // own c-prefetch copies
   tc_fence_after();
   if (tid == 0) phase_mark(p, 2);
   const int q = warp & 3;
@@ -1093,6 +1161,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int j = tid % U;
     const int u = unit0 + j;
     const float4 bias = *reinterpret_cast<const float4*>(p.bias + prow0 + j * G);
+    const float* cbuf = reinterpret_cast<const float*>(base + p.cbuf_off);
     for (int cl = tid / U; cl < my_cols; cl += 2 * ew) {
       const int nit = (cl + ew < my_cols) ? 2 : 1;
       float4 v[2][kMaxS];
@@ -1106,7 +1175,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int s = 0; s < kMaxS; ++s)
             if (s < S) v[h][s] = ld_cluster_v4(peer[s] + off);
           r[h] = rtab[c_lo + cl + h * ew];
-          cin[h] = (r[h].flags & ROW_FIRST) ? 0.f : p.c_pool[r[h].slot * H + u];
+          cin[h] = cbuf[(cl + h * ew) * U + j];
         }
       }
 #pragma unroll
@@ -1238,7 +1307,7 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   a.xkb = env_xkb > 0 ? env_xkb : 4;
   while (a.xkb > 1 && nk % a.xkb != 0) a.xkb >>= 1;
   int xstage = nhalf * 128 * a.xkb;
-  const int budget = smem - 1024 - kTailBytes;
+  const int budget = smem - 1024 - kTailBytes - ((((cpb + S - 1) / S) * a.U * 4 + 1023) & ~1023);
   if (nk * 16 * 1024 + 2 * xstage <= budget && nk <= 8) a.wcb = nk / 2;  // whole slice resident
   if (env_wcb > 0) a.wcb = env_wcb;
   int stages = (budget - kWRing * a.wcb * 16 * 1024) / xstage;
@@ -1247,7 +1316,8 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   a.xring = stages * xstage;
   const int region = kWRing * a.wcb * 16 * 1024 + a.xring;
   const int pbytes = cpb * 128 * 4;
-  const size_t need = 1024 + kTailBytes + (region > pbytes ? region : pbytes);
+  a.cbuf_off = kTailBytes + (region > pbytes ? region : pbytes);
+  const size_t need = 1024 + a.cbuf_off + ((((cpb + S - 1) / S) * a.U * 4 + 1023) & ~1023);
   if (need > static_cast<size_t>(smem)) return cudaSuccess;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(2 * S, tiles / 2, nblk);

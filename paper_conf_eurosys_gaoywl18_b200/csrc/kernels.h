@@ -81,6 +81,7 @@ struct StepArgs {
   int* dead;                  // [n_slots] 1 once the slot's request emitted <eos> (ROW_EOS rows
                               // are then no-ops); cleared by the request's first encoder step
   int* eos_host;              // host-mapped [max_requests]: decode step + 1 of the <eos>, or 0
+  int pchunk;                 // split-K exchange chunk (columns), 0 = whole tile (BM_PCHUNK)
   int cbuf_off;               // set by the launcher: shared-memory offset (from the 1 KB-aligned
                               // base) of the epilogue's prefetched c-state rows
 };
