@@ -88,6 +88,13 @@ typedef struct {
                              /* L427-L437; chain requests only)                            */
   int bucket_width;          /* graph batching: bucket i holds lengths (i*w, (i+1)*w] and */
                              /* its graph is unrolled to (i+1)*w steps (L427, L631); 10    */
+  int workers;               /* Algorithm 1 workers of this engine (§4, §8f N2), one */
+                             /* stream each on the engine's device; Schedule(worker) runs */
+                             /* for each idle worker, FormBatchedTask skips subgraphs     */
+                             /* pinned to another worker (Alg. 1 line 27, L381). 1 =      */
+                             /* request sharding's one worker per GPU (default). >1 needs */
+                             /* policy CELLULAR and persistent 0; the bf16 LSTM launches  */
+                             /* then use a <= 113 KB plan so two workers' CTAs share SMs. */
 } bm_config;
 
 enum {
@@ -98,7 +105,7 @@ enum {
 
 /* Fill *cfg with defaults: device 0, BF16, WALL, hidden 1024, 1 layer, 65536 slots,
  * 65536 requests, MaxTasksToSubmit 5, Min 1, k 0, max_decode_len 512, keep_results 0,
- * record_log 1, persistent 0, policy BM_POLICY_CELLULAR, bucket_width 10. */
+ * record_log 1, persistent 0, policy BM_POLICY_CELLULAR, bucket_width 10, workers 1. */
 void bm_config_default(bm_config* cfg);
 
 /* ---------------------------------------------------------------- cells (bm_load_cell) */
@@ -228,6 +235,7 @@ typedef struct {
   double tick;     /* submit time (tick or seconds)                                       */
   int first_row;   /* index into the rows array returned by bm_read_log_rows             */
   int n_rows;
+  int worker;      /* Algorithm 1 worker that ran the task (bm_config.workers)            */
 } bm_task_record;
 
 typedef struct {

@@ -129,7 +129,7 @@ class Replay:
 
     def __init__(self, cell_types: Sequence[Tuple[int, int]], max_slots: int = 1 << 20,
                  max_tasks_to_submit: int = 5, min_followon: int = 1,
-                 schedule_when_outstanding_leq: int = 0):
+                 schedule_when_outstanding_leq: int = 0, workers: int = 1):
         # cell_types: list of (bmax, priority); cell id = position
         self.cts = [CellType(i, bm, pr) for i, (bm, pr) in enumerate(cell_types)]
         self.pool = SlotPool(max_slots)
@@ -138,10 +138,13 @@ class Replay:
         self.k = schedule_when_outstanding_leq
         self.reqs: List[Req] = []
         self.tasks: List[Task] = []
-        self.inflight: deque = deque()
+        # one manager, W workers (§4, Alg. 1): each worker runs its own tasks in order,
+        # one tick per task; workers run in parallel (§8f N2 on one device)
+        self.W = workers
+        self.inflight_w: List[deque] = [deque() for _ in range(workers)]
         self.completions: List[Tuple[int, float]] = []   # (rid, tick) in completion order
         self.now = 0.0
-        self.last_finish = 0.0
+        self.last_finish_w = [0.0] * workers
 
     # ------------------------------------------------------------ request processor (A1)
     def admit(self, kind: int, cells: Sequence[int], length: int = 0, decode_len: int = 0,
@@ -384,23 +387,26 @@ class Replay:
         t = 0.0
         while True:
             self.now = t
-            while self.inflight and self.inflight[0].finish <= t:
-                self.retire(self.inflight.popleft())
+            # S21 with W workers: retire every task finishing by t in (finish, worker) order
+            while True:
+                due = [(q[0].finish, w) for w, q in enumerate(self.inflight_w) if q and q[0].finish <= t]
+                if not due:
+                    break
+                self.retire(self.inflight_w[min(due)[1]].popleft())
             while pending and requests[pending[0]]["arrival"] <= t:
                 i = pending.pop(0)
                 q = requests[i]
                 rid_of[i] = self.admit(q["kind"], q["cells"], q.get("length", 0),
                                        q.get("decode_len", 0), q.get("left"), q.get("right"),
                                        q.get("eos_step"))
-            if len(self.inflight) <= self.k:
-                for task in self.schedule(0):
-                    start = max(t, self.last_finish)
-                    task.finish = start + 1
-                    self.last_finish = task.finish
-                    self.inflight.append(task)
-            cand = []
-            if self.inflight:
-                cand.append(self.inflight[0].finish)
+            for w in range(self.W):   # Schedule(worker) for every idle worker, in id order
+                if len(self.inflight_w[w]) <= self.k:
+                    for task in self.schedule(w):
+                        start = max(t, self.last_finish_w[w])
+                        task.finish = start + 1
+                        self.last_finish_w[w] = task.finish
+                        self.inflight_w[w].append(task)
+            cand = [q[0].finish for q in self.inflight_w if q]
             if pending:
                 cand.append(requests[pending[0]]["arrival"])
             if not cand:

@@ -36,7 +36,7 @@ class Config(C.Structure):
         "device", "precision", "clock", "hidden", "pool_layers", "max_slots", "max_requests",
         "max_tasks_to_submit", "min_followon_batch", "schedule_when_outstanding_leq",
         "max_decode_len", "keep_results", "record_logits", "time_kernels", "record_log",
-        "persistent", "policy", "bucket_width")]
+        "persistent", "policy", "bucket_width", "workers")]
 
 
 class CellDesc(C.Structure):
@@ -69,7 +69,7 @@ class Result(C.Structure):
 
 class TaskRecord(C.Structure):
     _fields_ = [("task", C.c_int), ("cell", C.c_int), ("tick", C.c_double),
-                ("first_row", C.c_int), ("n_rows", C.c_int)]
+                ("first_row", C.c_int), ("n_rows", C.c_int), ("worker", C.c_int)]
 
 
 class RowRecord(C.Structure):
@@ -331,7 +331,7 @@ class Engine:
             t = tasks[i]
             rr = [(int(rows[j].req_id), rows[j].node, rows[j].slot)
                   for j in range(t.first_row, t.first_row + t.n_rows)]
-            out.append({"task": t.task, "cell": t.cell, "tick": t.tick, "rows": rr})
+            out.append({"task": t.task, "cell": t.cell, "tick": t.tick, "rows": rr, "worker": t.worker})
         return out
 
     # ---------------------------------------------------------------- direct cell access

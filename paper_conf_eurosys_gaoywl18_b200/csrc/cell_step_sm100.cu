@@ -768,9 +768,15 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   // 128-row LSTM / projection tiles keep a 128 KB weight slice + a 64 KB activation ring)
   static const int env_xkb = getenv("BM_XKB") ? atoi(getenv("BM_XKB")) : 0;
   a.xkb = 1;
+  // two workers share the SMs (small_plan): 2 x 16 KB weight chunks, a <= 64 KB activation
+  // ring and 128-column exchange chunks keep a CTA under half an SM's shared memory
+  // (measured with two engines, tools/dual_bench.py)
+  const bool small = a.small_plan && EPI == EPI_LSTM && env_wcb == 0;
+  if (small) a.wcb = 1;
   if (!internal && EPI != EPI_LEAF) {
     if (npad <= 64) a.xkb = 4, a.xring = 2 * 4 * npad * 128;
     else if (npad <= 128) a.xkb = 2, a.xring = 2 * 2 * npad * 128;
+    else if (small) a.xring = 32 * 1024;
     else if (env_wcb == 0) a.xkb = 2, a.wcb = 2, a.xring = 2 * 2 * npad * 128;  // 64 KB weight ring
   }
   if (env_xkb > 0) a.xkb = env_xkb;
@@ -784,7 +790,8 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   const int S = EPI == EPI_PROJ ? 1 : a.S;
   // epilogue c-state prefetch: ceil(cols / S) columns x 128 B (LSTM 32 units, internal 2 x 16)
   static const int env_pchunk = getenv("BM_PCHUNK") ? atoi(getenv("BM_PCHUNK")) : 0;
-  a.pchunk = (EPI != EPI_PROJ && env_pchunk > 0 && env_pchunk % 64 == 0 && env_pchunk < npad) ? env_pchunk : 0;
+  const int pchunk = env_pchunk > 0 ? env_pchunk : (a.small_plan && EPI == EPI_LSTM ? 128 : 0);
+  a.pchunk = (EPI != EPI_PROJ && pchunk > 0 && pchunk % 64 == 0 && pchunk < npad) ? pchunk : 0;
   const int cbuf_bytes = (EPI == EPI_LSTM || EPI == EPI_INTERNAL) && a.pchunk == 0
                              ? (((cols + S - 1) / S) * (EPI == EPI_INTERNAL ? 2 : 1) * a.U * 4 + 1023) & ~1023
                              : 0;
@@ -1350,7 +1357,7 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
 cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st) {
   if (a.b <= 0) return cudaSuccess;
   static const int use_pair = getenv("BM_PAIR") ? atoi(getenv("BM_PAIR")) : 1;
-  if (use_pair && a.epi == EPI_LSTM) {  // CTA-pair path (falls through if not eligible)
+  if (use_pair && a.epi == EPI_LSTM && !a.small_plan) {  // CTA-pair path (falls through if not eligible)
     bool done = false;
     cudaError_t e = rows_host != nullptr ? (a.b <= kMaxRowsInline ? launch_pair<true>(a, rows_host, st, &done)
                                                                    : cudaSuccess)

@@ -154,6 +154,26 @@ struct Task {
   std::vector<RowDesc> desc; // device row descriptors, built at submission (A3)
   int ev_first = -1, ev_count = 0;  // timed launches (time_kernels)
   std::vector<int> batch_reqs;      // graph batching: the batch's requests (on its last task)
+  int worker = 0;                   // Algorithm 1 worker (bm_config.workers)
+};
+
+// Launch state of one Algorithm-1 worker (§4, §8f N2): its stream, in-progress queue,
+// completion counter, launch chain and per-launch device scratch. The Engine's own copies of
+// these fields (stream, inflight, launched, ...) are the ACTIVE worker's; select_worker()
+// swaps them with the parked copies, so the launch / retire code serves any worker.
+struct WorkerState {
+  cudaStream_t stream = nullptr;
+  std::deque<Task> inflight;
+  uint64_t launched = 0;
+  double last_finish = 0;
+  unsigned long long* signal_host = nullptr;
+  unsigned long long* signal_dev = nullptr;
+  unsigned int* dep_flag = nullptr;
+  unsigned int dep_seq = 0;
+  bool pdl_ok = false;
+  unsigned int* sig_ctas = nullptr;
+  unsigned int* done_ctas = nullptr;
+  unsigned long long* amax = nullptr;
 };
 
 struct TimedLaunch {
@@ -245,7 +265,13 @@ struct Engine {
   std::vector<int> tl_b;
   uint64_t tl_n = 0;
 
+  // workers (§8f N2): parked launch state of the inactive workers; `cur` is active
+  std::vector<WorkerState> parked;
+  int cur = 0;
+  uint64_t tasks_total = 0;         // tasks over all workers (task log index)
+
   bool device() const { return cfg.clock != BM_CLOCK_DRY; }
+  std::deque<Task>& inflight_of(int w) { return w == cur ? inflight : parked[w].inflight; }
   size_t elem() const { return cfg.precision == BM_PREC_BF16 ? 2 : 4; }
   size_t H() const { return static_cast<size_t>(cfg.hidden); }
   void* h_layer(int l) const {
@@ -256,12 +282,13 @@ struct Engine {
 
 // scheduler.cpp
 bm_status admit_request(Engine& e, int ri);
-int schedule(Engine& e, std::vector<Task>& out);     // Schedule(worker 0): tasks formed
+int schedule(Engine& e, int worker, std::vector<Task>& out);  // Schedule(worker): tasks formed
 void retire_task(Engine& e, Task& t);
 bool has_ready(const Engine& e);
 void slot_release(Engine& e, int s);
 
 // runtime.cpp
+void select_worker(Engine& e, int w);
 bm_status launch_tasks(Engine& e, std::vector<Task>& tasks);
 double wall_now(const Engine& e);
 

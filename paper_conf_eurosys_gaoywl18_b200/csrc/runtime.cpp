@@ -68,6 +68,30 @@ void algo_cost(const Engine& e, const Cell& c, int b, bool proj, double* bytes, 
 
 }  // namespace
 
+// ---------------------------------------------------------------- workers (§8f N2)
+static void swap_active(Engine& e, WorkerState& w) {
+  std::swap(e.stream, w.stream);
+  std::swap(e.inflight, w.inflight);
+  std::swap(e.launched, w.launched);
+  std::swap(e.last_finish, w.last_finish);
+  std::swap(e.signal_host, w.signal_host);
+  std::swap(e.signal_dev, w.signal_dev);
+  std::swap(e.dep_flag, w.dep_flag);
+  std::swap(e.dep_seq, w.dep_seq);
+  std::swap(e.pdl_ok, w.pdl_ok);
+  std::swap(e.sig_ctas, w.sig_ctas);
+  std::swap(e.done_ctas, w.done_ctas);
+  std::swap(e.amax, w.amax);
+}
+
+// Make worker w's launch state the engine's active one (no-op with one worker).
+void select_worker(Engine& e, int w) {
+  if (w == e.cur || e.parked.empty()) return;
+  swap_active(e, e.parked[e.cur]);
+  swap_active(e, e.parked[w]);
+  e.cur = w;
+}
+
 // ---------------------------------------------------------------- launching tasks
 static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, const RowDesc* rows_host,
                                  int b, int layer, bool proj, int* ev_out, unsigned long long* signal) {
@@ -102,6 +126,7 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
   a.tok = e.tok;
   a.dead = e.dead;
   a.eos_host = e.eos_dev;
+  a.small_plan = e.cfg.workers > 1 ? 1 : 0;  // two workers' CTAs share the SMs
   a.W = proj ? c.W_out : c.W[layer];
   a.bias = proj ? c.b_out : c.bias[layer];
   a.W_rows = proj ? c.d.vocab : c.G * e.cfg.hidden;
@@ -218,9 +243,11 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
       t.finish = start + 1.0;
       e.last_finish = t.finish;
     }
+    const uint64_t task_index = e.tasks_total++;
     if (e.cfg.record_log) {
       bm_task_record rec;
-      rec.task = static_cast<int>(t.seq);
+      rec.task = static_cast<int>(task_index);
+      rec.worker = e.cur;
       rec.cell = t.ct;
       rec.tick = t.tick;
       rec.first_row = static_cast<int>(e.log_rows.size());
@@ -316,17 +343,17 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
   return BM_OK;
 }
 
-// Retire every in-flight task the device has finished (and, on the virtual clock, whose tick
-// has come). Returns the number retired.
-static int retire_ready(Engine& e, bool block) {
-  int n = 0;
-  while (!e.inflight.empty()) {
+// Retire the active worker's oldest in-flight task if the device has finished it (and, on the
+// virtual clock, its tick has come). Returns 1 if retired.
+static int retire_front(Engine& e, bool block) {
+  if (e.inflight.empty()) return 0;
+  {
     Task& t = e.inflight.front();
-    if (e.cfg.clock != BM_CLOCK_WALL && t.finish > e.now) break;
+    if (e.cfg.clock != BM_CLOCK_WALL && t.finish > e.now) return 0;
     if (e.device()) {
       volatile unsigned long long* sig = e.signal_host;
       if (*sig <= t.seq) {
-        if (!block && e.cfg.clock == BM_CLOCK_WALL) break;
+        if (!block && e.cfg.clock == BM_CLOCK_WALL) return 0;
         while (*sig <= t.seq) {
         }
       }
@@ -349,7 +376,39 @@ static int retire_ready(Engine& e, bool block) {
     }
     e.inflight.pop_front();
     e.stats.retire_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
-    ++n;
+  }
+  return 1;
+}
+
+// Retire every finished in-flight task of every worker. Virtual clock: in (finish tick,
+// worker) order (S21 with W workers, as the replay); wall clock: each worker's FIFO.
+static int retire_ready(Engine& e, bool block) {
+  int n = 0;
+  const int W = e.cfg.workers;
+  if (W == 1) {
+    while (retire_front(e, block)) ++n;
+    return n;
+  }
+  if (e.cfg.clock != BM_CLOCK_WALL) {
+    for (;;) {
+      int best = -1;
+      double bf = 0;
+      for (int w = 0; w < W; ++w) {
+        const std::deque<Task>& q = e.inflight_of(w);
+        if (!q.empty() && q.front().finish <= e.now && (best < 0 || q.front().finish < bf)) {
+          best = w;
+          bf = q.front().finish;
+        }
+      }
+      if (best < 0) break;
+      select_worker(e, best);
+      n += retire_front(e, block);
+    }
+  } else {
+    for (int w = 0; w < W; ++w) {
+      select_worker(e, w);
+      while (retire_front(e, block)) ++n;
+    }
   }
   return n;
 }
@@ -362,13 +421,29 @@ static void admit_due(Engine& e) {
   }
 }
 
+static bm_status schedule_and_launch_one(Engine& e, int* n_tasks);
+
+// Schedule(worker) for every idle worker, in id order (Alg. 1: "whenever some worker becomes
+// idle", L371; S19 idle = <= k outstanding tasks).
 static bm_status schedule_and_launch(Engine& e, int* n_tasks) {
+  *n_tasks = 0;
+  for (int w = 0; w < e.cfg.workers; ++w) {
+    select_worker(e, w);
+    int n = 0;
+    bm_status s = schedule_and_launch_one(e, &n);
+    if (s != BM_OK) return s;
+    *n_tasks += n;
+  }
+  return BM_OK;
+}
+
+static bm_status schedule_and_launch_one(Engine& e, int* n_tasks) {
   *n_tasks = 0;
   if (static_cast<int>(e.inflight.size()) > e.cfg.schedule_when_outstanding_leq) return BM_OK;
   static thread_local std::vector<Task> tasks;
   tasks.clear();
   const auto t0 = std::chrono::steady_clock::now();
-  schedule(e, tasks);
+  schedule(e, e.cur, tasks);
   e.stats.sched_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
   e.stats.schedule_calls += 1;
   if (tasks.empty()) return BM_OK;
@@ -381,8 +456,10 @@ static bm_status schedule_and_launch(Engine& e, int* n_tasks) {
   return BM_OK;
 }
 
-static bool all_done(const Engine& e) {
-  return e.pending.empty() && e.inflight.empty() && !has_ready(e);
+static bool all_done(Engine& e) {
+  for (int w = 0; w < e.cfg.workers; ++w)
+    if (!e.inflight_of(w).empty()) return false;
+  return e.pending.empty() && !has_ready(e);
 }
 
 // One round of the virtual-time event loop (S21); advances the clock to the next event.
@@ -392,7 +469,8 @@ static bm_status virtual_round(Engine& e, int* n_tasks) {
   bm_status s = schedule_and_launch(e, n_tasks);
   if (s != BM_OK) return s;
   double next = 1e300;
-  if (!e.inflight.empty()) next = std::min(next, e.inflight.front().finish);
+  for (int w = 0; w < e.cfg.workers; ++w)
+    if (!e.inflight_of(w).empty()) next = std::min(next, e.inflight_of(w).front().finish);
   if (!e.pending.empty()) next = std::min(next, e.reqs[e.pending.front()].t_arrival);
   if (next == 1e300) return all_done(e) ? BM_E_AGAIN : BM_E_STATE;  // nothing can progress
   e.now = next;
@@ -442,6 +520,7 @@ void bm_config_default(bm_config* c) {
   c->persistent = 0;
   c->policy = BM_POLICY_CELLULAR;
   c->bucket_width = 10;
+  c->workers = 1;
 }
 
 static void dump_timeline(Engine& e) {
@@ -461,6 +540,19 @@ static void dump_timeline(Engine& e) {
 }
 
 static void free_device(Engine& e) {
+  select_worker(e, 0);
+  for (size_t w = 1; w < e.parked.size(); ++w) {
+    WorkerState& ws = e.parked[w];
+    if (ws.stream) {
+      cudaStreamSynchronize(ws.stream);
+      cudaStreamDestroy(ws.stream);
+    }
+    if (ws.signal_host) cudaFreeHost(ws.signal_host);
+    cudaFree(ws.dep_flag);
+    cudaFree(ws.sig_ctas);
+    cudaFree(ws.done_ctas);
+    cudaFree(ws.amax);
+  }
   if (!e.device()) return;
   dump_timeline(e);
   cudaFree(e.tl_dev);
@@ -515,7 +607,8 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       c.max_slots < 1 || c.max_requests < 1 || c.max_requests >= (1 << 23) ||
       c.max_tasks_to_submit < 1 || c.min_followon_batch < 1 || c.schedule_when_outstanding_leq < 0 ||
       c.max_decode_len < 1 || c.precision < 0 || c.precision > 1 || c.clock < 0 || c.clock > 2 ||
-      c.policy < 0 || c.policy > 1 || c.bucket_width < 1)
+      c.policy < 0 || c.policy > 1 || c.bucket_width < 1 || c.workers < 1 || c.workers > 8 ||
+      (c.workers > 1 && c.policy != BM_POLICY_CELLULAR))
     return BM_E_INVAL;
   Engine* e = new (std::nothrow) Engine();
   if (e == nullptr) return BM_E_NOMEM;
@@ -524,6 +617,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
   e->free_slots_heap.resize(c.max_slots);
   for (int i = 0; i < c.max_slots; ++i) e->free_slots_heap[i] = i;  // sorted == valid min-heap
   e->t0 = std::chrono::steady_clock::now();
+  if (c.workers > 1) e->parked.resize(c.workers);
   if (e->device()) {
     Engine& E = *e;
     auto fail = [&](bm_status s) {
@@ -615,6 +709,24 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       E.tl_host.assign(Engine::kTimeline, 0);
       E.tl_retire.assign(Engine::kTimeline, 0);
       E.tl_b.assign(Engine::kTimeline, 0);
+    }
+    // workers 1..W-1 (§8f N2): own stream, completion counter, launch chain, device scratch
+    for (int w = 1; w < c.workers; ++w) {
+      WorkerState& ws = E.parked[w];
+      if (cudaStreamCreateWithFlags(&ws.stream, cudaStreamNonBlocking) != cudaSuccess ||
+          cudaHostAlloc(reinterpret_cast<void**>(&ws.signal_host), sizeof(unsigned long long),
+                        cudaHostAllocMapped) != cudaSuccess)
+        return fail(BM_E_NOMEM);
+      *ws.signal_host = 0;
+      if (cudaHostGetDevicePointer(reinterpret_cast<void**>(&ws.signal_dev), ws.signal_host, 0) != cudaSuccess ||
+          dalloc(&ws.dep_flag, 1) != cudaSuccess || dalloc(&ws.sig_ctas, 1) != cudaSuccess ||
+          dalloc(&ws.done_ctas, 1) != cudaSuccess || dalloc(&ws.amax, 512) != cudaSuccess)
+        return fail(BM_E_NOMEM);
+      if (cudaMemsetAsync(ws.dep_flag, 0, 4, E.stream) != cudaSuccess ||
+          cudaMemsetAsync(ws.sig_ctas, 0, 4, E.stream) != cudaSuccess ||
+          cudaMemsetAsync(ws.done_ctas, 0, 4, E.stream) != cudaSuccess ||
+          cudaMemsetAsync(ws.amax, 0, 512 * 8, E.stream) != cudaSuccess)
+        return fail(BM_E_CUDA);
     }
     if (cudaStreamSynchronize(E.stream) != cudaSuccess) return fail(BM_E_CUDA);
   }
@@ -849,6 +961,7 @@ bm_status bm_schedule_step(bm_engine* h, int* n_tasks) {
   } else {
     s = virtual_round(e, &n);
   }
+  select_worker(e, 0);
   if (n_tasks) *n_tasks = n;
   return s;
 }
@@ -859,6 +972,7 @@ bm_status bm_poll(bm_engine* h, bm_completion* out, int cap, int* n) {
   if (e.cfg.clock == BM_CLOCK_WALL) {
     e.now = wall_now(e);
     retire_ready(e, false);
+    select_worker(e, 0);
   }
   const int k = std::min<int>(cap, static_cast<int>(e.completions.size()));
   if (k > 0) memcpy(out, e.completions.data(), k * sizeof(bm_completion));
@@ -868,7 +982,9 @@ bm_status bm_poll(bm_engine* h, bm_completion* out, int cap, int* n) {
 }
 
 static bool persistent_eligible(const Engine& e) {
-  if (!e.cfg.persistent || !e.device() || e.cfg.precision != BM_PREC_BF16 || e.cells.size() != 1) return false;
+  if (!e.cfg.persistent || !e.device() || e.cfg.precision != BM_PREC_BF16 || e.cells.size() != 1 ||
+      e.cfg.workers != 1)
+    return false;
   const Cell& c = e.cells[0];
   const int K = c.K0 + c.K1;
   return c.d.kind == BM_CELL_LSTM && c.d.layers == 1 && c.S >= 1 && c.S <= 4 && c.kslice <= 512 &&
@@ -988,6 +1104,7 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
       admit_due(e);
       s = schedule_and_launch(e, &n);
       if (s != BM_OK) {
+        select_worker(e, 0);
         persistent_stop(e);
         return s;
       }
@@ -997,6 +1114,7 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
     while ((s = virtual_round(e, &n)) == BM_OK) {
     }
     if (s != BM_E_AGAIN) {
+      select_worker(e, 0);
       persistent_stop(e);
       return s;
     }
@@ -1005,7 +1123,13 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
     s = persistent_stop(e);
     if (s != BM_OK) return s;
   }
-  if (e.device()) CK(cudaStreamSynchronize(e.stream));
+  if (e.device()) {
+    for (int w = e.cfg.workers - 1; w >= 0; --w) {
+      select_worker(e, w);
+      CK(cudaStreamSynchronize(e.stream));
+    }
+  }
+  select_worker(e, 0);
   if (n_completed) *n_completed = static_cast<int>(e.completions.size() - before);
   return BM_OK;
 }

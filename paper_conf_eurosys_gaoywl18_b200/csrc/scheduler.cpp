@@ -276,6 +276,7 @@ Task submit(Engine& e, int ct, int worker, const std::vector<Cand>& batch) {
   Task t;
   t.ct = ct;
   t.tick = e.now;
+  t.worker = worker;
   t.rows.reserve(batch.size());
   t.desc.reserve(batch.size());
   Cell& c = e.cells[ct];
@@ -394,9 +395,8 @@ static int schedule_graph(Engine& e, std::vector<Task>& out) {
 
 // Schedule(worker), Alg. 1 lines 4-11. If the chosen type forms no task only because the
 // slot pool is exhausted, fall through to the next choice [S22].
-int schedule(Engine& e, std::vector<Task>& out) {
+int schedule(Engine& e, int worker, std::vector<Task>& out) {
   if (e.cfg.policy == BM_POLICY_GRAPH) return schedule_graph(e, out);
-  const int worker = 0;
   const int nc = static_cast<int>(e.cells.size());
   uint64_t excluded = 0;
   for (int attempt = 0; attempt < nc; ++attempt) {

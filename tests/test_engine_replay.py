@@ -57,6 +57,7 @@ def _compare(e, rp):
     for a, t in zip(log, rp.tasks):
         assert a["cell"] == t.ct
         assert a["tick"] == t.tick
+        assert a["worker"] == t.worker
         assert a["rows"] == [(r.rid, r.node, r.slot) for r in t.rows]
     comp = e.poll()
     assert [(c.req_id, c.t_done) for c in comp] == [(rid, float(tk)) for rid, tk in rp.completions]
@@ -189,3 +190,26 @@ def test_eos_request_rejected_when_invalid():
         e.submit(bm.REQ_SEQ2SEQ, ids[0], ids[1], [3, 4], 0, decode_len=4, eos_id=128)  # >= vocab
     with pytest.raises(RuntimeError):
         e.submit(bm.REQ_SEQ2SEQ, ids[0], ids[1], [3, 4], 0, decode_len=4, eos_id=-2)
+
+
+@settings(max_examples=150, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 100_000), n=st.integers(1, 20),
+       bmax=st.lists(st.integers(1, 6), min_size=5, max_size=5),
+       prio=st.permutations([0, 1, 2, 3, 4]), max_tasks=st.integers(1, 5),
+       k=st.integers(0, 3), slots=st.integers(4, 40), workers=st.integers(2, 4),
+       kinds=st.sampled_from([[CHAIN], [SEQ2SEQ], [TREE], [CHAIN, SEQ2SEQ, TREE]]), eos=st.booleans())
+def test_multi_worker_traces_bit_exact(seed, n, bmax, prio, max_tasks, k, slots, workers, kinds, eos):
+    """§8f N2: one manager, W workers (L317): Schedule(worker) for each idle worker, subgraphs
+    pinned to the worker running them (Alg. 1 lines 21, 27; unpinned at in-flight 0, L381).
+    The engine (W streams) and the replay agree task for task, worker for worker."""
+    reqs = _random_reqs(seed, n, kinds, eos=eos)
+    need = max((len(q["left"]) if q["kind"] == TREE else 1) for q in reqs)
+    slots = max(slots, need)
+    kinds_c = [bm.CELL_LSTM, bm.CELL_LSTM, bm.CELL_LSTM_PROJ, bm.CELL_TREE_LEAF, bm.CELL_TREE_INTERNAL]
+    e, _ = _engine(list(zip(kinds_c, bmax, prio)), max_slots=slots, max_requests=64,
+                   max_tasks_to_submit=max_tasks, schedule_when_outstanding_leq=k, workers=workers)
+    _submit_all(e, reqs)
+    e.run()
+    rp = Replay(list(zip(bmax, prio)), max_slots=slots, max_tasks_to_submit=max_tasks,
+                schedule_when_outstanding_leq=k, workers=workers).run(reqs)
+    _compare(e, rp)

@@ -259,3 +259,67 @@ def test_graph_batching_policy_h1024(prec):
         hs, cs = cells.chain_lstm(w, q.tokens)
         assert np.max(np.abs(r["h"][0] - hs[0])) <= TOL[prec]
         assert np.max(np.abs(r["c"][0] - cs[0])) <= TOL[prec]
+
+
+@pytest.mark.parametrize("prec", [bm.PREC_BF16, bm.PREC_FP32])
+def test_two_workers_chain_h1024(prec):
+    """§8f N2 on one device: two Algorithm-1 workers (two streams, subgraphs pinned to the worker
+    running them, L317/L381). Virtual clock: the task log (worker included) equals the replay
+    with W = 2; every request's final state matches the oracle."""
+    trace = gen.chain_trace(48, 2048, seed=1001, rate=3.0)
+    e, cid, w = lstm_engine(1024, 1, 2048, prec, bmax=512, clock=bm.CLOCK_VIRTUAL, max_slots=256,
+                            max_requests=256, keep_results=1, schedule_when_outstanding_leq=2, workers=2)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    e.run()
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": q.arrival, "length": q.length} for q in trace]
+    rp = Replay([(512, 0)], max_slots=256, schedule_when_outstanding_leq=2, workers=2).run(reqs)
+    assert {t.worker for t in rp.tasks} == {0, 1}
+    _check_log(e, rp)
+    worst = 0.0
+    for i, q in enumerate(trace):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, q.tokens)
+        worst = max(worst, np.max(np.abs(r["h"][0] - hs[0])), np.max(np.abs(r["c"][0] - cs[0])))
+    assert worst <= TOL[prec], worst
+
+
+def test_two_workers_seq2seq_eos():
+    """Two workers with the Seq2Seq decoder (projection scratch per worker) and <eos> stop."""
+    h, V, L = 64, 256, 4
+    trace = _s2s_trace(V, 12, 99)
+    kw = dict(bmax=(512, 256), clock=bm.CLOCK_VIRTUAL, max_slots=64, max_requests=64, keep_results=1,
+              max_decode_len=40, workers=2)
+    e, (ce, cd), (enc, dec) = seq2seq_engine(h, L, V, bm.PREC_BF16, **kw)
+    eos = 7
+    for toks, T, t in trace:
+        e.submit(bm.REQ_SEQ2SEQ, ce, cd, toks, t, decode_len=T, eos_id=eos)
+    e.run()
+    steps = []
+    for i, (toks, T, _) in enumerate(trace):
+        r = e.read_result(i, L, decode_len=T)
+        y = [int(v) for v in r["tokens"]]
+        m = y.index(-1) if -1 in y else T
+        steps.append(m - 1 if (m < T or y[T - 1] == eos) else None)
+        o = cells.seq2seq(enc, dec, toks, T, forced_tokens=y[:m], eos_id=eos)
+        for l in range(L):
+            assert np.max(np.abs(r["h"][l] - o["h"][l])) <= TOL[bm.PREC_BF16]
+    reqs = [{"kind": SEQ2SEQ, "cells": [0, 1], "arrival": t, "length": len(toks), "decode_len": T,
+             "eos_step": steps[i]} for i, (toks, T, t) in enumerate(trace)]
+    _check_log(e, Replay([(512, 0), (256, 1)], max_slots=64, workers=2).run(reqs))
+
+
+def test_two_workers_wall_clock():
+    """Two workers on the wall clock (the bench path): all requests complete, sampled results
+    match the oracle."""
+    trace = gen.chain_trace(400, 1024, seed=6, rate=200000.0)
+    e, cid, w = lstm_engine(1024, 1, 1024, bm.PREC_BF16, bmax=512, max_slots=1024, max_requests=1024,
+                            keep_results=1, schedule_when_outstanding_leq=2, workers=2)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    assert e.run() == 400
+    assert sorted(c.req_id for c in e.poll()) == list(range(400))
+    for i in (0, 123, 399):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, trace[i].tokens)
+        assert np.max(np.abs(r["h"][0] - hs[0])) <= TOL[bm.PREC_BF16]

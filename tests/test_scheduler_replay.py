@@ -267,3 +267,57 @@ def test_n1_eos_invariants(seed, n, bmax, max_tasks, k):
             assert e < m <= q["decode_len"]
             t_eos = next(task.finish for task, s in dec if s == e)
             assert all(task.tick < t_eos for task, _ in dec)
+
+
+
+# ---------------------------------------------------------------- §8f N2: several workers
+@settings(max_examples=200, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 100_000), n=st.integers(1, 16), bmax=st.integers(1, 6),
+       max_tasks=st.integers(1, 5), k=st.integers(0, 3), workers=st.integers(1, 4))
+def test_n2_pinning_invariants(seed, n, bmax, max_tasks, k, workers):
+    """Algorithm 1 with W workers (L345-L381): every node runs once; each worker runs its tasks
+    one at a time; a subgraph never has nodes in flight on two workers at once (it is pinned to
+    the worker that runs it until its in-flight count drops to 0, lines 21/27, L381); a task
+    holds nodes of ready subgraphs only (dependencies as with one worker)."""
+    rng = np.random.default_rng(seed)
+    reqs, t = [], 0.0
+    for _ in range(n):
+        t += float(rng.integers(0, 3))
+        if rng.random() < 0.5:
+            reqs.append({"kind": CHAIN, "cells": [0], "arrival": t, "length": int(rng.integers(1, 9))})
+        else:
+            reqs.append({"kind": SEQ2SEQ, "cells": [0, 1], "arrival": t, "length": int(rng.integers(1, 5)),
+                         "decode_len": int(rng.integers(1, 6))})
+    rp = Replay([(bmax, 0), (bmax, 1)], max_tasks_to_submit=max_tasks, schedule_when_outstanding_leq=k,
+                workers=workers).run(reqs)
+    seen = set()
+    for task in rp.tasks:
+        for row in task.rows:
+            assert (row.rid, row.node) not in seen
+            seen.add((row.rid, row.node))
+    assert len(seen) == sum(q["length"] + q.get("decode_len", 0) for q in reqs)
+    for w in range(workers):
+        mine = sorted((t_.tick, t_.finish) for t_ in rp.tasks if t_.worker == w)
+        for (a0, a1), (b0, b1) in zip(mine, mine[1:]):
+            assert b1 >= a1 + 1          # one task per tick per worker
+    # pinning: intervals [tick, finish) of one subgraph's tasks on different workers are disjoint
+    spans = {}
+    for task in rp.tasks:
+        for row in task.rows:
+            r = rp.reqs[row.rid]
+            sg = r.node_sg[row.node]
+            spans.setdefault(id(sg), []).append((task.tick, task.finish, task.worker))
+    for lst in spans.values():
+        for i, (s0, f0, w0) in enumerate(lst):
+            for s1, f1, w1 in lst[i + 1:]:
+                if w0 != w1:
+                    assert f0 <= s1 or f1 <= s0
+    # a chain's steps run in order: step v+1's task is submitted no earlier than step v's
+    for rid, r in enumerate(rp.reqs):
+        ticks = {}
+        for task in rp.tasks:
+            for row in task.rows:
+                if row.rid == rid:
+                    ticks[row.node] = (task.tick, task.finish, task.index)
+        for v in range(1, len(ticks)):
+            assert ticks[v][2] > ticks[v - 1][2]
