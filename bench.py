@@ -71,6 +71,8 @@ def parse():
                    help="graph: the padding + bucketing graph-batching baseline of §7.1 (L427: bucket "
                         "width 10, round robin over buckets) on the same kernels (lstm workload only)")
     p.add_argument("--bucket-width", type=int, default=10)
+    p.add_argument("--workers", type=int, default=1,
+                   help="Algorithm 1 workers per GPU (one stream each, subgraph pinning, §8f N2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--out", default="")
@@ -126,12 +128,12 @@ def weight_arrays(w):
 
 # ------------------------------------------------------------------------------ engine
 def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, keep=0, persistent=0,
-                 policy=0, bucket_width=10):
+                 policy=0, bucket_width=10, workers=1):
     h, L, V = WL[wl]["hidden"], WL[wl]["layers"], WL[wl]["vocab"]
     e = bm.Engine(device=device, hidden=h, pool_layers=L, max_slots=1 << 16, max_requests=max_requests,
                   schedule_when_outstanding_leq=lookahead, time_kernels=time_kernels, keep_results=keep,
                   max_decode_len=340, record_log=0, persistent=persistent, policy=policy,
-                  bucket_width=bucket_width)
+                  bucket_width=bucket_width, workers=workers)
     if wl == "lstm":
         c = w["cell"]
         cid = e.load_cell(bm.CELL_LSTM, L, V, 512, 0, c.W, c.b, c.E)
@@ -335,7 +337,7 @@ def main():
     if dist is not None:
         shard.broadcast_arrays(weight_arrays(w), dist, device=torch.device("cuda", local))
     e, cells = build_engine(bm, wl, w, local, max_requests=max(n_req, 1 << 15) + 64, lookahead=a.lookahead,
-                            persistent=a.persistent, policy=policy, bucket_width=a.bucket_width)
+                            persistent=a.persistent, policy=policy, workers=a.workers, bucket_width=a.bucket_width)
     stream = torch.cuda.ExternalStream(e.stream(), device=torch.device("cuda", local))
 
     def barrier():
@@ -413,7 +415,7 @@ def main():
     # ---- e2e: public API with host buffers (submit from host, descriptors H2D every Schedule
     #      call inside bm_run, final h rows D2H), timed on the host clock around the whole thing
     e2, cells2 = build_engine(bm, wl, w, local, max_requests=n_req + 64, lookahead=a.lookahead,
-                              time_kernels=0, keep=1, persistent=a.persistent, policy=policy,
+                              time_kernels=0, keep=1, persistent=a.persistent, policy=policy, workers=a.workers,
                               bucket_width=a.bucket_width)
     L, H = WL[wl]["layers"], WL[wl]["hidden"]
     hbuf = torch.empty((n_req, L, H), dtype=torch.float32).pin_memory().numpy()
@@ -453,7 +455,10 @@ def main():
         t_kern = st["timed_ms"]
         timing = ("CUDA events on the engine stream around a sample of cell-step launches (every 8th: "
                   "events between launches would disable PDL overlap)")
-        kernel = "cell_step_sm100_kernel<EPI_LSTM>"
+        kernel = {"lstm": "LSTM cell step: cell_pair_kernel (257-512 rows) + cell_step_sm100_kernel<EPI_LSTM>",
+                  "seq2seq": "Seq2Seq cell steps: 4 LSTM layers (cell_pair_kernel / cell_step_sm100_kernel<EPI_LSTM>) "
+                             "+ projection/argmax cell_step_sm100_kernel<EPI_PROJ>",
+                  "tree": "TreeLSTM cell steps: cell_step_sm100_kernel<EPI_LEAF> + <EPI_INTERNAL>"}[wl]
     else:                    # persistent kernel: tasks run inside one launch
         t_kern = st["span_ms"]
         timing = ("persistent kernel: per-task device span (%globaltimer, first CTA ready .. last CTA "
@@ -488,7 +493,7 @@ def main():
                            "saturation_burst_rate_per_gpu": mu, "lookahead_k": a.lookahead,
                            "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
                                  "step (serving)", "parallelism": f"request-sharded x{world}",
-                           "persistent_kernel": bool(a.persistent),
+                           "persistent_kernel": bool(a.persistent), "workers_per_gpu": a.workers,
                            "policy": ("cellular batching (Algorithm 1)" if policy == bm.POLICY_CELLULAR else
                                       f"graph-batching baseline: padding + bucketing, width {a.bucket_width}, "
                                       "round robin over buckets (L427)")},

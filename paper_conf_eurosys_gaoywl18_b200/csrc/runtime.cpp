@@ -32,13 +32,17 @@ double wall_now(const Engine& e) {
 
 namespace {
 
-#define CK(x)                         \
-  do {                                \
-    cudaError_t err__ = (x);          \
-    if (err__ != cudaSuccess) {       \
-      e.sticky_cuda = true;           \
-      return BM_E_CUDA;               \
-    }                                 \
+// A failing CUDA call makes the engine unusable (BM_E_CUDA is sticky, include/bm.h); the
+// failing call and the CUDA error are reported on stderr once.
+#define CK(x)                                                                                  \
+  do {                                                                                         \
+    cudaError_t err__ = (x);                                                                   \
+    if (err__ != cudaSuccess) {                                                                \
+      if (!e.sticky_cuda)                                                                      \
+        fprintf(stderr, "bm: %s:%d: %s -> %s\n", __FILE__, __LINE__, #x, cudaGetErrorString(err__)); \
+      e.sticky_cuda = true;                                                                    \
+      return BM_E_CUDA;                                                                        \
+    }                                                                                          \
   } while (0)
 
 template <class T>
@@ -220,7 +224,10 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const 
     int ev = -1;
     bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, 0, true, &ev, fused ? signal : nullptr);
     if (s != BM_OK) return s;
-    if (t && ev >= 0) t->ev_count += 1;
+    if (t && ev >= 0) {
+      if (t->ev_first < 0) t->ev_first = ev;  // the projection may be the task's only timed launch
+      t->ev_count += 1;
+    }
   }
   if (signal != nullptr && !fused) {
     CK(launch_signal(signal, e.stream));
@@ -366,7 +373,9 @@ static int retire_front(Engine& e, bool block) {
       for (int k = 0; k < t.ev_count; ++k) {
         TimedLaunch& tl = e.ev_pool[(t.ev_first + k) % e.ev_pool.size()];
         float ms = 0;
-        if (cudaEventElapsedTime(&ms, tl.beg, tl.end) == cudaSuccess) {
+        if (cudaEventElapsedTime(&ms, tl.beg, tl.end) != cudaSuccess) {
+          cudaGetLastError();  // not sticky: must not leak into a later launch's error check
+        } else {
           e.stats.timed_launches += 1;
           e.stats.timed_ms += ms;
           e.stats.timed_bytes += tl.bytes;
