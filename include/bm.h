@@ -224,7 +224,8 @@ bm_status bm_release(bm_engine* e, uint64_t req_id);
 
 /* Bulk result read for the consecutive ids [first_id, first_id + n), all completed and kept:
  * one device->host copy per contiguous table range. h: [n][pool_layers][hidden] fp32 or
- * NULL; tokens: [n][max_decode_len] or NULL. Then releases them if release != 0. */
+ * NULL; tokens: [n][max_decode_len] or NULL (entries past a request's last emitted token are
+ * -1). Then releases them if release != 0. */
 bm_status bm_read_results_many(bm_engine* e, uint64_t first_id, int n, float* h, int32_t* tokens,
                                int release);
 

@@ -1210,6 +1210,14 @@ bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh
     done += len;
   }
   CK(cudaStreamSynchronize(e.stream));
+  if (toks) {  // as bm_read_result: after an <eos> (N1) the remaining entries are -1
+    for (int i = 0; i < n; ++i) {
+      const Request& r = e.reqs[(first_id + i) % R];
+      if (r.kind != BM_REQ_SEQ2SEQ) continue;
+      const int T = r.eos_step >= 0 ? r.eos_step + 1 : r.n_nodes - r.enc_len;
+      for (size_t s = T; s < D; ++s) toks[i * D + s] = -1;
+    }
+  }
   if (release) {
     for (int i = 0; i < n; ++i) {
       Request& r = e.reqs[(first_id + i) % R];

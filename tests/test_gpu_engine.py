@@ -164,6 +164,13 @@ def test_seq2seq_eos_terminated(prec, h, V, n):
             assert np.max(np.abs(r["h"][l] - o["h"][l])) <= tol
             assert np.max(np.abs(r["c"][l] - o["c"][l])) <= tol
     assert steps[0] == j
+    # the bulk read reports the same tokens, -1 after each request's last emitted one
+    bulk = np.zeros((n, 40), np.int32)
+    e.read_results_many(0, n, tokens=bulk, release=False)
+    for i, (toks, T, _) in enumerate(trace):
+        m = (steps[i] + 1) if steps[i] is not None else T
+        one = e.read_result(i, L, decode_len=T)["tokens"]
+        assert list(bulk[i, :T]) == list(one) and (bulk[i, m:] == -1).all()
     reqs = [{"kind": SEQ2SEQ, "cells": [0, 1], "arrival": t, "length": len(toks), "decode_len": T,
              "eos_step": steps[i]} for i, (toks, T, t) in enumerate(trace)]
     _check_log(e, Replay([(512, 0), (256, 1)], max_slots=64).run(reqs))
