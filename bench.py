@@ -477,6 +477,12 @@ def main():
             "avg_rows_per_task": st["rows"] / max(1, st["tasks"]), "tensor_tflops": tflops,
             "tensor_frac": tflops / bf16_peak,
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)" if peaks else "fallback 6.65 TB/s",
+            # the same sampled launches timed on the device (%globaltimer: first CTA past its
+            # dependency wait .. last CTA done): excludes the serialisation the events impose
+            "device_span_us": (st["span_ms"] * 1e3 / st["span_launches"]) if st["span_launches"] else None,
+            "frac_device_span": ((st["timed_bytes"] / max(1, st["timed_launches"])) /
+                                 (st["span_ms"] / 1e3 / st["span_launches"]) / 1e9 / hbm)
+            if st["span_launches"] and st["timed_ms"] > 0 else None,
             "note": ("algorithmic bytes count the 16.8 MB weight stream per step even when the persistent "
                      "kernel keeps the weights on chip (so frac can exceed what DRAM moved)")}
     cpu = None
