@@ -8,6 +8,7 @@
 #include <stdint.h>
 
 #include "kernels.h"
+#include "sm100_ptx.cuh"
 
 namespace bm {
 namespace {
@@ -305,9 +306,9 @@ __global__ void convert_kernel(const float* __restrict__ src, void* dst, size_t 
 
 // Completion signal (§5): one thread bumps the counter that the host polls through
 // zero-copy pinned memory; system-scope release so the host sees everything before it.
-__global__ void signal_kernel(unsigned long long* counter) {
+__global__ void signal_kernel(unsigned long long* counter, unsigned long long value) {
   __threadfence_system();
-  atomicAdd_system(counter, 1ull);
+  ptx::signal_store(counter, value);
 }
 
 __global__ void pool_io_kernel(void* h_pool, float* c_pool, const int32_t* slots, int n, int H,
@@ -367,8 +368,8 @@ cudaError_t launch_convert(const float* src, void* dst, size_t n, int bf16, cuda
   return cudaGetLastError();
 }
 
-cudaError_t launch_signal(unsigned long long* counter, cudaStream_t st) {
-  signal_kernel<<<1, 1, 0, st>>>(counter);
+cudaError_t launch_signal(unsigned long long* counter, unsigned long long value, cudaStream_t st) {
+  signal_kernel<<<1, 1, 0, st>>>(counter, value);
   return cudaGetLastError();
 }
 

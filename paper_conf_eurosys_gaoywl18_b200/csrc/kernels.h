@@ -65,6 +65,7 @@ struct StepArgs {
                               // fill), bit 2: no weight copies; results are garbage
   // launch path
   unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
+  unsigned long long sig_value;  // the counter value this task's completion publishes (seq + 1)
   unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)
   int pdl;                    // launch with programmatic dependent launch (overlap setup)
   int cpb;                    // CTA-pair kernel: batch columns per column block
@@ -110,6 +111,7 @@ struct PersistArgs {
   unsigned int* gbar;         // grid-barrier counter (zero at launch)
   int* err;                   // set to 1 if the kernel aborted (host stopped feeding)
   unsigned long long* signal; // host-mapped completion counter
+  unsigned long long sig_base;   // counter value before the run's first task
   unsigned long long* span;   // optional: 64 task-start slots (time_kernels)
   unsigned long long* span_acc;
   unsigned long long* phase;  // diagnostics (BM_PHASE_DUMP): per-CTA timestamps of task 20
@@ -136,7 +138,7 @@ cudaError_t launch_pack_tiles(const float* src, void* dst, int G, int H, int K, 
                               int n_rows, cudaStream_t st);
 cudaError_t launch_convert(const float* src, void* dst, size_t n, int bf16, cudaStream_t st);
 // Completion signal (A12): bump a host-mapped counter after everything before it in stream.
-cudaError_t launch_signal(unsigned long long* counter, cudaStream_t st);
+cudaError_t launch_signal(unsigned long long* counter, unsigned long long value, cudaStream_t st);
 // Pool access helpers (tests): gather/scatter fp32 rows of h (bf16 or fp32) and c.
 cudaError_t launch_pool_io(void* h_pool, float* c_pool, const int32_t* slots, int n, int H,
                            float* h_buf, float* c_buf, int write, int bf16, cudaStream_t st);

@@ -98,7 +98,8 @@ void select_worker(Engine& e, int w) {
 
 // ---------------------------------------------------------------- launching tasks
 static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, const RowDesc* rows_host,
-                                 int b, int layer, bool proj, int* ev_out, unsigned long long* signal) {
+                                 int b, int layer, bool proj, int* ev_out, unsigned long long* signal,
+                                 unsigned long long sig_value = 0) {
   StepArgs a{};
   a.epi = proj ? EPI_PROJ : c.epi;
   a.G = proj ? 1 : c.G;
@@ -148,6 +149,7 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
   static const int experiment = getenv("BM_EXPERIMENT") ? atoi(getenv("BM_EXPERIMENT")) : 0;
   a.experiment = experiment;
   a.signal = signal;
+  a.sig_value = sig_value;
   a.sig_ctas = e.sig_ctas;
   // PDL only directly behind another tcgen05 launch: the chain flag orders launches among
   // themselves, while copies / other kernels before a launch need full stream ordering
@@ -209,11 +211,13 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const 
   const bool lstm = c.epi == EPI_LSTM;
   const bool proj = c.d.kind == BM_CELL_LSTM_PROJ;
   const bool fused = e.cfg.precision == BM_PREC_BF16;
+  const unsigned long long sig_value = t != nullptr ? t->seq + 1 : 0;  // completed-task count
   const int L = lstm ? c.d.layers : 1;
   for (int l = 0; l < L; ++l) {
     int ev = -1;
     const bool last = l == L - 1 && !proj;
-    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, l, false, &ev, (last && fused) ? signal : nullptr);
+    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, l, false, &ev, (last && fused) ? signal : nullptr,
+                                  sig_value);
     if (s != BM_OK) return s;
     if (t && ev >= 0) {
       if (t->ev_first < 0) t->ev_first = ev;
@@ -222,7 +226,7 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const 
   }
   if (proj) {
     int ev = -1;
-    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, 0, true, &ev, fused ? signal : nullptr);
+    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, 0, true, &ev, fused ? signal : nullptr, sig_value);
     if (s != BM_OK) return s;
     if (t && ev >= 0) {
       if (t->ev_first < 0) t->ev_first = ev;  // the projection may be the task's only timed launch
@@ -230,7 +234,7 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const 
     }
   }
   if (signal != nullptr && !fused) {
-    CK(launch_signal(signal, e.stream));
+    CK(launch_signal(signal, sig_value, e.stream));
     e.stats.kernel_launches += 1;
   }
   return BM_OK;
@@ -1035,6 +1039,7 @@ static bm_status persistent_start(Engine& e) {
   a.gbar = e.gbar;
   a.err = e.perr;
   a.signal = e.signal_dev;
+  a.sig_base = e.launched;  // == run_base below
   a.span = e.cfg.time_kernels ? e.spans : nullptr;
   a.span_acc = e.cfg.time_kernels ? e.spans + 128 : nullptr;
   static const char* dump = getenv("BM_PHASE_DUMP");
