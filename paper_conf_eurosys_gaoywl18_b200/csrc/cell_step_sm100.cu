@@ -133,12 +133,11 @@ __device__ __forceinline__ void launch_done(const StepArgs& p, unsigned int* cta
   if (atomicAdd(ctas, 1u) == total - 1) {
     *ctas = 0;
     __threadfence();
-    if (p.signal != nullptr) {  // before the chain flag: the next task's signal is causally later
+    if (p.dep_flag != nullptr) st_release_gpu(p.dep_flag, p.dep_seq);
+    if (p.signal != nullptr) {  // the task's own slot: no ordering against other tasks needed
       __threadfence_system();
       signal_store(p.signal, p.sig_value);
-      __threadfence_system();
     }
-    if (p.dep_flag != nullptr) st_release_gpu(p.dep_flag, p.dep_seq);
   }
 }
 
@@ -550,12 +549,11 @@ __global__ void __launch_bounds__(kThreads, 2)
       if (tid == 0) {
         *p.done_ctas = 0;
         __threadfence();
+        if (p.dep_flag != nullptr) st_release_gpu(p.dep_flag, p.dep_seq);
         if (p.signal != nullptr) {  // completion signal (A12) fused into the last CTA
           __threadfence_system();
           signal_store(p.signal, p.sig_value);
-          __threadfence_system();
         }
-        if (p.dep_flag != nullptr) st_release_gpu(p.dep_flag, p.dep_seq);
       }
     }
     if (tid == 0) phase_mark(p, 4);

@@ -65,7 +65,7 @@ struct StepArgs {
                               // fill), bit 2: no weight copies; results are garbage
   // launch path
   unsigned long long* signal; // non-null on a task's last launch: host-mapped completion counter
-  unsigned long long sig_value;  // the counter value this task's completion publishes (seq + 1)
+  unsigned long long sig_value;  // the value this task's completion publishes in *signal (seq + 1)
   unsigned int* sig_ctas;     // CTA counter for the fused signal (zero between launches)
   int pdl;                    // launch with programmatic dependent launch (overlap setup)
   int cpb;                    // CTA-pair kernel: batch columns per column block
@@ -89,6 +89,10 @@ struct StepArgs {
                               // base) of the epilogue's prefetched c-state rows
 };
 
+// Completion signals (A12): a ring of host-mapped slots; task `seq` of a worker writes seq + 1
+// into slot seq % kSignalSlots (one writer per slot at a time: kSignalSlots >> tasks in flight).
+constexpr int kSignalSlots = 256;
+
 // Persistent weight-stationary LSTM engine (lstm_persistent_sm100.cu).
 struct TaskHdr {
   int32_t seq;      // run-local task index; the kernel polls for the value it expects
@@ -110,8 +114,8 @@ struct PersistArgs {
   float* res_c;
   unsigned int* gbar;         // grid-barrier counter (zero at launch)
   int* err;                   // set to 1 if the kernel aborted (host stopped feeding)
-  unsigned long long* signal; // host-mapped completion counter
-  unsigned long long sig_base;   // counter value before the run's first task
+  unsigned long long* signal; // host-mapped completion slots [kSignalSlots]
+  unsigned long long sig_base;   // worker task index of the run's first task
   unsigned long long* span;   // optional: 64 task-start slots (time_kernels)
   unsigned long long* span_acc;
   unsigned long long* phase;  // diagnostics (BM_PHASE_DUMP): per-CTA timestamps of task 20

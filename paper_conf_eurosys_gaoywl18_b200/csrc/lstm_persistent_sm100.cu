@@ -362,8 +362,8 @@ __global__ void __launch_bounds__(kThreads, 1) lstm_persistent_kernel(const __gr
           atomicAdd(p.span_acc + 1, 1ull);
         }
         __threadfence_system();
-        signal_store(p.signal, p.sig_base + static_cast<unsigned long long>(t) + 1ull);  // A12
-        __threadfence_system();
+        const unsigned long long seq = p.sig_base + static_cast<unsigned long long>(t);
+        signal_store(p.signal + seq % kSignalSlots, seq + 1ull);  // completion signal (A12)
       }
     }
   }

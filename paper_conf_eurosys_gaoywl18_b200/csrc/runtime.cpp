@@ -211,7 +211,8 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const 
   const bool lstm = c.epi == EPI_LSTM;
   const bool proj = c.d.kind == BM_CELL_LSTM_PROJ;
   const bool fused = e.cfg.precision == BM_PREC_BF16;
-  const unsigned long long sig_value = t != nullptr ? t->seq + 1 : 0;  // completed-task count
+  const unsigned long long sig_value = t != nullptr ? t->seq + 1 : 0;  // this task's completion
+  if (signal != nullptr && t != nullptr) signal += t->seq % kSignalSlots;  // its own slot
   const int L = lstm ? c.d.layers : 1;
   for (int l = 0; l < L; ++l) {
     int ev = -1;
@@ -362,7 +363,8 @@ static int retire_front(Engine& e, bool block) {
     Task& t = e.inflight.front();
     if (e.cfg.clock != BM_CLOCK_WALL && t.finish > e.now) return 0;
     if (e.device()) {
-      volatile unsigned long long* sig = e.signal_host;
+      // the task's own signal slot (kSignalSlots-entry ring, written once per task)
+      volatile unsigned long long* sig = e.signal_host + (t.seq % kSignalSlots);
       if (*sig <= t.seq) {
         if (!block && e.cfg.clock == BM_CLOCK_WALL) return 0;
         while (*sig <= t.seq) {
@@ -666,10 +668,10 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
     if (cudaHostAlloc(reinterpret_cast<void**>(&E.ring_host), E.ring_rows * sizeof(RowDesc),
                       cudaHostAllocDefault) != cudaSuccess)
       return fail(BM_E_NOMEM);
-    if (cudaHostAlloc(reinterpret_cast<void**>(&E.signal_host), sizeof(unsigned long long),
+    if (cudaHostAlloc(reinterpret_cast<void**>(&E.signal_host), kSignalSlots * sizeof(unsigned long long),
                       cudaHostAllocMapped) != cudaSuccess)
       return fail(BM_E_NOMEM);
-    *E.signal_host = 0;
+    memset(E.signal_host, 0, kSignalSlots * sizeof(unsigned long long));
     // <eos> reports (N1): written by the projection kernel, read at retire
     if (cudaHostAlloc(reinterpret_cast<void**>(&E.eos_host), R * sizeof(int), cudaHostAllocMapped) != cudaSuccess ||
         cudaHostGetDevicePointer(reinterpret_cast<void**>(&E.eos_dev), E.eos_host, 0) != cudaSuccess)
@@ -727,10 +729,10 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
     for (int w = 1; w < c.workers; ++w) {
       WorkerState& ws = E.parked[w];
       if (cudaStreamCreateWithFlags(&ws.stream, cudaStreamNonBlocking) != cudaSuccess ||
-          cudaHostAlloc(reinterpret_cast<void**>(&ws.signal_host), sizeof(unsigned long long),
+          cudaHostAlloc(reinterpret_cast<void**>(&ws.signal_host), kSignalSlots * sizeof(unsigned long long),
                         cudaHostAllocMapped) != cudaSuccess)
         return fail(BM_E_NOMEM);
-      *ws.signal_host = 0;
+      memset(ws.signal_host, 0, kSignalSlots * sizeof(unsigned long long));
       if (cudaHostGetDevicePointer(reinterpret_cast<void**>(&ws.signal_dev), ws.signal_host, 0) != cudaSuccess ||
           dalloc(&ws.dep_flag, 1) != cudaSuccess || dalloc(&ws.sig_ctas, 1) != cudaSuccess ||
           dalloc(&ws.done_ctas, 1) != cudaSuccess || dalloc(&ws.amax, 512) != cudaSuccess)
