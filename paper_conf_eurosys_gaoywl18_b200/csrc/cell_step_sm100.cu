@@ -899,7 +899,7 @@ __device__ __forceinline__ void cluster_wait() {
   asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-template <bool INL>
+template <bool INL, bool WCPA>
 __global__ void __launch_bounds__(kThreads, 1)
     cell_pair_kernel(const __grid_constant__ StepArgs p, const __grid_constant__ RowsParam<INL> rr) {
   extern __shared__ uint8_t smem_raw[];
@@ -925,7 +925,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int xkb = p.xkb > 0 ? p.xkb : 1;
   const int nst = nk / xkb;
   const int x_blk_bytes = nhalf * 128;
-  const int x_stage_bytes = x_blk_bytes * xkb;
+  // WCPA: each stage also carries this CTA's xkb weight K blocks (16 KB each), loaded by the
+  // producers' cp.async next to the activations (LSU path) instead of the TMA weight ring
+  const int x_stage_bytes = x_blk_bytes * xkb + (WCPA ? xkb * 16384 : 0);
   const int kStages = min(pairk::kStagesMax, max(2, p.xring / x_stage_bytes));
   const int wcb = p.wcb;
   const int kpc = min(wcb, nk);
@@ -945,7 +947,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);
   uint8_t* smem = base + kTailBytes;
   uint8_t* w_ring = smem;
-  uint8_t* x_st = smem + kWRing * wcb * wblk_bytes;
+  uint8_t* x_st = smem + (WCPA ? 0 : kWRing * wcb * wblk_bytes);
 
   if (tid == 0) phase_mark(p, 0);
   if (tid == 0) {
@@ -1025,6 +1027,14 @@ __global__ void __launch_bounds__(kThreads, 1)
             else cp_async_16(xs + dst_off[i], dummy, 0);  // zero fill (h0 = 0, padding)
           }
         }
+        if constexpr (WCPA) {  // this CTA's pre-swizzled 16 KB weight tile of K block k
+          const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
+                                (static_cast<size_t>(tile) * ((p.K0 + p.K1) / kBK) + k / kBK) * wblk_bytes;
+          const uint32_t wdst = smem_u32(x_st + s * x_stage_bytes + xkb * x_blk_bytes + j * wblk_bytes);
+#pragma unroll
+          for (int i = 0; i < wblk_bytes / 16 / kProducerThreads; ++i)
+            cp_async_16(wdst + (tid + i * kProducerThreads) * 16, wsrc + (tid + i * kProducerThreads) * 16, 16);
+        }
       }
       if (st == 0) {
         const int cper_ = (ncols + p.S - 1) / p.S;
@@ -1037,7 +1047,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
-    if (lane == 0) {
+    if (!WCPA && lane == 0) {
       const int kblocks = (p.K0 + p.K1) / kBK;
       const uint8_t* wsrc =
           static_cast<const uint8_t*>(p.W) + (static_cast<size_t>(tile) * kblocks + k_begin / kBK) * wblk_bytes;
@@ -1076,7 +1086,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int kb = st * xkb + j;
         const int c = kb / kpc;
         const int ws = c % kWRing;
-        if (kb % kpc == 0) {
+        if (!WCPA && kb % kpc == 0) {
           const uint32_t wpar = (c / kWRing) & 1;
           if (lane == 0) {
             wait_bounded<false>(wfull0 + 8 * ws, wpar);
@@ -1088,11 +1098,12 @@ __global__ void __launch_bounds__(kThreads, 1)
           tc_fence_after();
         }
         if (lane == 0) {
-          const uint64_t a = sdesc_sw128(smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
+          const uint64_t a = sdesc_sw128(WCPA ? smem_u32(x_st + s * x_stage_bytes + xkb * x_blk_bytes + j * wblk_bytes)
+                                              : smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
           const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes + j * x_blk_bytes));
 #pragma unroll
           for (int k = 0; k < kBK / 16; ++k) mma_bf16_pair(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
-          if (kb % kpc == kpc - 1 || kb == nk - 1) mma_commit_pair(wempty0 + 8 * ws, pair_mask);
+          if (!WCPA && (kb % kpc == kpc - 1 || kb == nk - 1)) mma_commit_pair(wempty0 + 8 * ws, pair_mask);
         }
         __syncwarp();
       }
@@ -1117,7 +1128,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         mbar_arrive_remote(pfull_l + 8 * s);
         for (int j = 0; j < xkb; ++j) {
           const int kb = st * xkb + j;
-          if (kb % kpc == 0) {
+          if (!WCPA && kb % kpc == 0) {
             const int c = kb / kpc;
             const int ws = c % kWRing;
             wait_bounded<false>(wfull0 + 8 * ws, (c / kWRing) & 1);
@@ -1255,9 +1266,13 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   static int max_clusters8 = 0;
   const int smem = 227 * 1024;
   if (state == 0) {
-    cudaError_t e = cudaFuncSetAttribute(cell_pair_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(cell_pair_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(cell_pair_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      e = cudaFuncSetAttribute(cell_pair_kernel<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(cell_pair_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(cell_pair_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) {
       state = -1;
       cudaGetLastError();
@@ -1274,7 +1289,7 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    if (cudaOccupancyMaxActiveClusters(&max_clusters8, cell_pair_kernel<false>, &cfg) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveClusters(&max_clusters8, cell_pair_kernel<false, false>, &cfg) != cudaSuccess) {
       max_clusters8 = 0;
       cudaGetLastError();
     }
@@ -1310,13 +1325,18 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   // stages of xkb K blocks
   static const int env_wcb = getenv("BM_PAIR_WCB") ? atoi(getenv("BM_PAIR_WCB")) : 0;
   static const int env_xkb = getenv("BM_PAIR_XKB") ? atoi(getenv("BM_PAIR_XKB")) : 0;
+  // weights by cp.async in the activation stages (default): the per-SM TMA engine completes
+  // bulk copies one at a time, the LSU path keeps more bytes in flight (-10% per step at
+  // b = 288..512, tools/kbench.py); BM_PAIR_WCPA=0 restores the TMA weight ring
+  static const int wcpa = getenv("BM_PAIR_WCPA") ? atoi(getenv("BM_PAIR_WCPA")) : 1;
   a.wcb = 2;
-  a.xkb = env_xkb > 0 ? env_xkb : 4;
+  a.xkb = env_xkb > 0 ? env_xkb : (wcpa ? 2 : 4);
   while (a.xkb > 1 && nk % a.xkb != 0) a.xkb >>= 1;
-  int xstage = nhalf * 128 * a.xkb;
+  int xstage = nhalf * 128 * a.xkb + (wcpa ? 16384 * a.xkb : 0);
+  if (wcpa) a.wcb = 0;  // no TMA weight ring
   const int budget = smem - 1024 - kTailBytes - ((((cpb + S - 1) / S) * a.U * 4 + 1023) & ~1023);
-  if (nk * 16 * 1024 + 2 * xstage <= budget && nk <= 8) a.wcb = nk / 2;  // whole slice resident
-  if (env_wcb > 0) a.wcb = env_wcb;
+  if (!wcpa && nk * 16 * 1024 + 2 * xstage <= budget && nk <= 8) a.wcb = nk / 2;  // whole slice resident
+  if (!wcpa && env_wcb > 0) a.wcb = env_wcb;
   int stages = (budget - kWRing * a.wcb * 16 * 1024) / xstage;
   stages = stages > pairk::kStagesMax ? pairk::kStagesMax : stages;
   if (stages < 2) return cudaSuccess;
@@ -1346,9 +1366,11 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
     memcpy(inline_rows.r, rows_host, sizeof(RowDesc) * a.b);
     a.rows = nullptr;
     a.rows_flag = nullptr;
-    return cudaLaunchKernelEx(&cfg, cell_pair_kernel<true>, a, inline_rows);
+    return wcpa ? cudaLaunchKernelEx(&cfg, cell_pair_kernel<true, true>, a, inline_rows)
+                : cudaLaunchKernelEx(&cfg, cell_pair_kernel<true, false>, a, inline_rows);
   } else {
-    return cudaLaunchKernelEx(&cfg, cell_pair_kernel<false>, a, RowsParam<false>{0});
+    return wcpa ? cudaLaunchKernelEx(&cfg, cell_pair_kernel<false, true>, a, RowsParam<false>{0})
+                : cudaLaunchKernelEx(&cfg, cell_pair_kernel<false, false>, a, RowsParam<false>{0});
   }
 }
 
