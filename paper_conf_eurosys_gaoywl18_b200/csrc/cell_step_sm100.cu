@@ -264,7 +264,11 @@ __global__ void __launch_bounds__(kThreads, 2)
   // (every mbarrier hand-off costs ~0.15-0.3 us of latency on the MMA's path, tools/pipe_bench.cu)
   const int xkb = p.xkb > 0 ? p.xkb : 1;
   const int nst = nk / xkb;
-  const int kStages = p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad * xkb, p.xring))
+  // wcpa (LSTM): the stage also carries the weight K blocks (loaded by the producers)
+  const bool wcpa = EPI == EPI_LSTM && p.wcpa != 0;
+  const int wblk_ = (EPI == EPI_PROJ ? 128 : G * U) * 128;
+  const int kStages = wcpa ? max(2, min(kMaxStages, p.xring / ((npad * 128 + wblk_) * xkb)))
+                    : p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad * xkb, p.xring))
                                        : x_stages_for(npad * xkb, p.xring);
   const int wcb = p.wcb;                                  // ring slot capacity in K blocks
   const int kpc = min(wcb, nk);                           // K blocks per weight chunk
@@ -283,9 +287,9 @@ __global__ void __launch_bounds__(kThreads, 2)
   RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);  // this CTA's rows (col0 + c)
   uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
   uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
-  uint8_t* x_st = smem + kWRing * wcb * wblk_bytes;       // kStages x xkb x npad x 128 B
+  uint8_t* x_st = smem + (wcpa ? 0 : kWRing * wcb * wblk_bytes);  // kStages x stage
   const int x_blk_bytes = npad * 128;                     // one K block of the activation tile
-  const int x_stage_bytes = x_blk_bytes * xkb;
+  const int x_stage_bytes = x_blk_bytes * xkb + (wcpa ? wblk_bytes * xkb : 0);
 
   // ---- setup (overlaps the previous launch's tail under PDL: touches no dependent data)
   if (tid == 0) phase_mark(p, 0);
@@ -390,6 +394,13 @@ __global__ void __launch_bounds__(kThreads, 2)
             }
           }
         }
+        if (wcpa) {  // this K block's pre-swizzled weight tile (16 KB), 4 x 16 B per thread
+          const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
+                                (static_cast<size_t>(blockIdx.y) * ((p.K0 + p.K1) / kBK) + k / kBK) * wblk_bytes;
+          const uint32_t wdst = smem_u32(x_st + s * x_stage_bytes + xkb * x_blk_bytes + j * wblk_bytes);
+          for (int i = tid; i < wblk_bytes / 16; i += kProducerThreads)
+            cp_async_16(wdst + i * 16, wsrc + i * 16, 16);
+        }
       }
       if (st == 0 && EPI != EPI_PROJ && p.pchunk == 0) {
         const int cper_ = (ncols + p.S - 1) / p.S;
@@ -403,7 +414,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
     // Weights are read-only: streaming starts before griddepcontrol.wait (PDL overlap).
-    if (lane == 0) {
+    if (!wcpa && lane == 0) {
       const int kblocks = (p.K0 + p.K1) / kBK;
       const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
                             (static_cast<size_t>(blockIdx.y) * kblocks + k_begin / kBK) * wblk_bytes;
@@ -442,7 +453,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         const int kb = st * xkb + j;
         const int c = kb / kpc;
         const int ws = c % kWRing;
-        if (kb % kpc == 0) {
+        if (!wcpa && kb % kpc == 0) {
           mbar_wait_warp(wfull0 + 8 * ws, (c / kWRing) & 1);
           tc_fence_after();
           if (lane == 0 && c < 4) phase_mark(p, 28 + c);  // weight chunk c at the MMA
@@ -450,7 +461,8 @@ __global__ void __launch_bounds__(kThreads, 2)
         }
         if (lane == 0) {
           const uint64_t a =
-              sdesc_sw128(smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
+              sdesc_sw128(wcpa ? smem_u32(x_st + s * x_stage_bytes + xkb * x_blk_bytes + j * wblk_bytes)
+                               : smem_u32(w_ring + ws * wcb * wblk_bytes + (kb % kpc) * wblk_bytes));
           const uint64_t b = sdesc_sw128(smem_u32(x_st + s * x_stage_bytes + j * x_blk_bytes));
           if (!(p.experiment & 8)) {  // diagnostics bit 8: no MMA instructions
 #pragma unroll
@@ -458,7 +470,7 @@ __global__ void __launch_bounds__(kThreads, 2)
               mma_bf16(tmem, a + 2 * k, b + 2 * k, idesc, (kb | k) != 0 ? 1u : 0u);
             }
           }
-          if (kb % kpc == kpc - 1 || kb == nk - 1) mma_commit(wempty0 + 8 * ws);
+          if (!wcpa && (kb % kpc == kpc - 1 || kb == nk - 1)) mma_commit(wempty0 + 8 * ws);
         }
         __syncwarp();
       }
@@ -780,6 +792,16 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
     else if (env_wcb == 0) a.xkb = 2, a.wcb = 2, a.xring = 2 * 2 * npad * 128;  // 64 KB weight ring
   }
   if (env_xkb > 0) a.xkb = env_xkb;
+  // BM_WCPA=1: LSTM weights by cp.async inside the activation stages (as the CTA-pair kernel),
+  // stages of xkb K blocks of (activations + 16 KB weights). Off by default here: this kernel's
+  // 128 KB K slice already moves in two 64 KB bulk copies and the two plans measure the same
+  // (tools/kbench.py, b = 16..256, within +-2%); the pair kernel's 32 KB chunks gain 10%.
+  static const int env_wcpa = getenv("BM_WCPA") ? atoi(getenv("BM_WCPA")) : 0;
+  a.wcpa = (EPI == EPI_LSTM && env_wcpa && !a.small_plan && env_wcb == 0) ? 1 : 0;
+  if (a.wcpa) {
+    a.xkb = npad <= 64 ? 4 : 2;
+    if (env_xkb > 0) a.xkb = env_xkb;
+  }
   const int nk_all = a.kslice / kBK;
   if (EPI == EPI_PROJ) {
     if (a.xkb > 1 && (a.H / kBK) % a.xkb != 0) a.xkb = 1;
@@ -795,7 +817,20 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   const int cbuf_bytes = (EPI == EPI_LSTM || EPI == EPI_INTERNAL) && a.pchunk == 0
                              ? (((cols + S - 1) / S) * (EPI == EPI_INTERNAL ? 2 : 1) * a.U * 4 + 1023) & ~1023
                              : 0;
-  a.cbuf_off = kTailBytes + region_bytes(a.pchunk > 0 ? a.pchunk : npad, a.wcb, a.xring, wblk, a.xkb, npad);
+  if (a.wcpa) {
+    const int stage = (npad * 128 + wblk) * a.xkb;
+    const int budget = 227 * 1024 - 1024 - kTailBytes - cbuf_bytes;
+    const int stages = std::min(kMaxStages, budget / stage);
+    if (stages < 2) {
+      a.wcpa = 0;  // does not fit: keep the TMA ring plan computed above
+    } else {
+      a.xring = stages * stage;
+      const int ptile = 129 * (a.pchunk > 0 ? a.pchunk : npad) * 4 + 4 * 128 * 4;
+      a.cbuf_off = kTailBytes + std::max(a.xring, ptile);
+    }
+  }
+  if (!a.wcpa)
+    a.cbuf_off = kTailBytes + region_bytes(a.pchunk > 0 ? a.pchunk : npad, a.wcb, a.xring, wblk, a.xkb, npad);
   const size_t smem = 1024 + a.cbuf_off + cbuf_bytes;
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;
