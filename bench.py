@@ -455,7 +455,7 @@ def main():
         t_kern = st["timed_ms"]
         timing = ("CUDA events on the engine stream around a sample of cell-step launches (every 8th: "
                   "events between launches would disable PDL overlap)")
-        kernel = {"lstm": "LSTM cell step: cell_pair_kernel (257-512 rows) + cell_step_sm100_kernel<EPI_LSTM>",
+        kernel = {"lstm": "LSTM cell step: cell_pair_kernel (129-512 rows) + cell_step_sm100_kernel<EPI_LSTM>",
                   "seq2seq": "Seq2Seq cell steps: 4 LSTM layers (cell_pair_kernel / cell_step_sm100_kernel<EPI_LSTM>) "
                              "+ projection/argmax cell_step_sm100_kernel<EPI_PROJ>",
                   "tree": "TreeLSTM cell steps: cell_step_sm100_kernel<EPI_LEAF> + <EPI_INTERNAL>"}[wl]

@@ -1333,9 +1333,10 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   if (state < 0) return cudaSuccess;
   const int K = a.K0 + a.K1;
   const int tiles = a.H / a.U;
-  // measured (tools/pair_sweep.sh, kbench spans): the pair kernel wins above 256 rows (b = 384:
-  // 23.3 vs 25.7 us) and loses below (b = 64: 17 vs 12 us) -- BM_PAIR_MIN overrides the cut
-  static const int min_b = getenv("BM_PAIR_MIN") ? atoi(getenv("BM_PAIR_MIN")) : 257;
+  // measured (tools/kbench.py, cp.async weights): the pair kernel wins from 129 rows up (b =
+  // 160 / 192 / 256: 19.4 / 19.9 / 21.0 vs 20.1 / 21.2 / 23.5 us), ties at 128 and loses below
+  // (b = 64: 17.9 vs 16.4 us) -- BM_PAIR_MIN overrides the cut
+  static const int min_b = getenv("BM_PAIR_MIN") ? atoi(getenv("BM_PAIR_MIN")) : 129;
   if (a.epi != EPI_LSTM || a.U != 32 || tiles % 2 != 0 || K % 1024 != 0 || a.b > 512 || a.b < min_b)
     return cudaSuccess;
   static const int env_s = getenv("BM_PAIR_S") ? atoi(getenv("BM_PAIR_S")) : 0;
