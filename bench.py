@@ -313,12 +313,21 @@ def main():
     import torch
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # one GPU per rank (NCCL over NVLink). With fewer GPUs than ranks (a functional check of the
+    # multi-rank path on one GPU) ranks share devices and the few collectives go over gloo.
+    ndev = max(1, torch.cuda.device_count())
+    local = local_rank % ndev
+    shared = world > ndev
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    coll_dev = None if shared else torch.device("cuda", local)
     from paper_conf_eurosys_gaoywl18_b200 import bm, shard
 
     wl = a.workload
@@ -335,7 +344,7 @@ def main():
     # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink), never again
     w = make_weights(wl)
     if dist is not None:
-        shard.broadcast_arrays(weight_arrays(w), dist, device=torch.device("cuda", local))
+        shard.broadcast_arrays(weight_arrays(w), dist, device=coll_dev)
     e, cells = build_engine(bm, wl, w, local, max_requests=max(n_req, 1 << 15) + 64, lookahead=a.lookahead,
                             persistent=a.persistent, policy=policy, workers=a.workers, bucket_width=a.bucket_width)
     stream = torch.cuda.ExternalStream(e.stream(), device=torch.device("cuda", local))
@@ -346,7 +355,7 @@ def main():
             dist.barrier()
 
     def allmax(x):
-        return shard.reduce_max(x, dist, device=torch.device("cuda", local))
+        return shard.reduce_max(x, dist, device=coll_dev)
 
     # ---- calibrate saturation: every request of a trace arrives at t = 0
     burst = make_trace(wl, n_req, None, seed=shard.rank_seed(7, rank))
@@ -407,7 +416,7 @@ def main():
             lats.append(comp["t_done"] - comp["t_arrival"])
     barrier()
     st = e.stats()
-    lat = shard.gather_samples(np.concatenate(lats), dist, device=torch.device("cuda", local))
+    lat = shard.gather_samples(np.concatenate(lats), dist, device=coll_dev)
     t_max = allmax(dev_ms / 1e3)
     total = n_req * a.steps * world
     value = total / t_max

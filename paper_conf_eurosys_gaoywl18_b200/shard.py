@@ -8,7 +8,8 @@ off the per-step path:
     gloo in the CPU tests),
   * max-over-ranks reductions of timings and a gather of latency samples at the end.
 The paper's own multi-GPU design (one manager, many workers, subgraph pinning and cross-GPU
-state migration, L317-L381) is SURVEY §8f row N2, not built here.
+state migration, L317-L381) is SURVEY §8f row N2: its workers and pinning are built inside one
+engine (bm_config.workers, one device); the cross-GPU migration is not.
 """
 from __future__ import annotations
 
