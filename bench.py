@@ -400,7 +400,7 @@ def main():
     barrier()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     dev_ms = 0.0
-    lats = []
+    lats, queue, compute = [], [], []
     with ClockSampler(local) as clk:
         for _ in range(a.steps):
             flush.zero_()
@@ -414,9 +414,13 @@ def main():
             dev_ms += ev0.elapsed_time(ev1)
             comp = e.poll_array(n_req + 16)
             lats.append(comp["t_done"] - comp["t_arrival"])
+            queue.append(comp["t_first"] - comp["t_arrival"])   # E5 (Fig. 9): queueing
+            compute.append(comp["t_done"] - comp["t_first"])     # ... and computation time
     barrier()
     st = e.stats()
     lat = shard.gather_samples(np.concatenate(lats), dist, device=coll_dev)
+    q_lat = shard.gather_samples(np.concatenate(queue), dist, device=coll_dev)
+    c_lat = shard.gather_samples(np.concatenate(compute), dist, device=coll_dev)
     t_max = allmax(dev_ms / 1e3)
     total = n_req * a.steps * world
     value = total / t_max
@@ -513,6 +517,10 @@ def main():
                                       f"graph-batching baseline: padding + bucketing, width {a.bucket_width}, "
                                       "round robin over buckets (L427)")},
                 "latency_ms": {"p50": p50 * 1e3, "p90": p90 * 1e3, "p99": p99 * 1e3},
+                # Fig. 9's decomposition (L597): queueing = arrival -> first node scheduled,
+                # computation = first node -> completion
+                "latency_split_ms": {k: dict(zip(("p50", "p90", "p99"), (x * 1e3 for x in shard.percentiles(v))))
+                                     for k, v in (("queueing", q_lat), ("computation", c_lat))},
                 "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu,
                 "clocks": clk.summary(), "gpu_launches": int(st["kernel_launches"]),
                 "sched_ns_per_task": st["sched_ns"] / max(1, st["tasks"])}
