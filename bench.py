@@ -71,6 +71,8 @@ def parse():
                    help="graph: the padding + bucketing graph-batching baseline of §7.1 (L427: bucket "
                         "width 10, round robin over buckets) on the same kernels (lstm workload only)")
     p.add_argument("--bucket-width", type=int, default=10)
+    p.add_argument("--lengths", default="wmt", choices=["wmt", "fixed24", "clip50", "clip100"],
+                   help="LSTM request lengths: WMT-like (configs[1]) or Fig. 11's variants (L643-L681)")
     p.add_argument("--workers", type=int, default=1,
                    help="Algorithm 1 workers per GPU (one stream each, subgraph pinning, §8f N2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -93,9 +95,22 @@ WL = {
 }
 
 
+LENGTHS = "wmt"   # --lengths (LSTM): wmt | fixed24 | clip50 | clip100 (Fig. 11)
+
+
+def chain_lengths(n, seed, kind):
+    """Fig. 11's length mixes: the WMT-like distribution, every request 24 steps, or WMT clipped
+    at 50 / 100 steps (L643-L667)."""
+    if kind == "fixed24":
+        return np.full(n, 24, np.int64)
+    wmt = gen.wmt_lengths(n, np.random.default_rng(seed + 77))
+    return np.minimum(wmt, {"clip50": 50, "clip100": 100}[kind])
+
+
 def make_trace(wl, n, rate, seed):
     if wl == "lstm":
-        return gen.chain_trace(n, WL[wl]["vocab"], seed, rate=rate)
+        lengths = None if LENGTHS == "wmt" else chain_lengths(n, seed, LENGTHS)
+        return gen.chain_trace(n, WL[wl]["vocab"], seed, rate=rate, lengths=lengths)
     if wl == "seq2seq":
         return gen.seq2seq_trace(n, WL[wl]["vocab"], seed, rate=rate)
     return gen.tree_trace(n, WL[wl]["vocab"], seed, rate=rate)
@@ -307,7 +322,9 @@ def reference_arm(a):
 
 # ------------------------------------------------------------------------------ main arm
 def main():
+    global LENGTHS
     a = parse()
+    LENGTHS = a.lengths if a.workload == "lstm" else "wmt"
     if a.impl == "reference":
         return reference_arm(a)
     import torch
@@ -498,6 +515,28 @@ def main():
             if st["span_launches"] and st["timed_ms"] > 0 else None,
             "note": ("algorithmic bytes count the 16.8 MB weight stream per step even when the persistent "
                      "kernel keeps the weights on chip (so frac can exceed what DRAM moved)")}
+    bound = None
+    if wl == "lstm" and LENGTHS == "fixed24":
+        # L679-L681: with every request 24 steps long the throughput bound is
+        # bmax / (24 x t_step(bmax)); t_step measured here on full 512-row tasks, back to back
+        rng = np.random.default_rng(5)
+        b = 512
+        slots = rng.choice(1 << 16, size=b, replace=False).astype(np.int32)
+        rows = np.stack([rng.integers(3, WL[wl]["vocab"], size=b), np.zeros(b), slots,
+                         (np.arange(b) % 2) * bm.ROW_PARITY], 1)
+        cid = cells[gen.CHAIN][0]
+        for _ in range(5):
+            e.cell_step(cid, rows, sync=False)
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for _ in range(50):
+            e.cell_step(cid, rows, sync=False)
+        ev1.record(stream)
+        ev1.synchronize()
+        t_step = ev0.elapsed_time(ev1) / 50 / 1e3
+        b_req = b / (24 * t_step) * world
+        bound = {"t_step_b512_us": t_step * 1e6, "bound_req_s": b_req, "fraction_of_bound": value / b_req,
+                 "paper": "BatchMaker at ~87% of 27,136 req/s on V100 (L679-L681)"}
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         cpu = cpu_oracle(wl, a.cpu_seconds)
@@ -505,7 +544,9 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": "requests/sec", "n_gpus": world, "steps": a.steps,
                 "warmup": a.warmup, "ms_per_step": t_max * 1e3 / a.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-                "config": {"workload": WL[wl]["config"], "requests_per_step": n_req,
+                "config": {"workload": WL[wl]["config"] if LENGTHS == "wmt" else
+                           WL[wl]["config"].replace("WMT-like lengths", f"Fig. 11 lengths '{LENGTHS}'"),
+                           "requests_per_step": n_req,
                            "offered_rate_per_gpu": lam_star, "p90_bound_ms": bound_ms,
                            "p90_bound_kind": bound_kind,
                            "max_offered_rate_under": bounds if a.rate <= 0 else None,
@@ -521,7 +562,7 @@ def main():
                 # computation = first node -> completion
                 "latency_split_ms": {k: dict(zip(("p50", "p90", "p99"), (x * 1e3 for x in shard.percentiles(v))))
                                      for k, v in (("queueing", q_lat), ("computation", c_lat))},
-                "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu,
+                "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu, "fixed_length_bound": bound,
                 "clocks": clk.summary(), "gpu_launches": int(st["kernel_launches"]),
                 "sched_ns_per_task": st["sched_ns"] / max(1, st["tasks"])}
         s = json.dumps(line)
