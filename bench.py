@@ -71,8 +71,9 @@ def parse():
                    help="graph: the padding + bucketing graph-batching baseline of §7.1 (L427: bucket "
                         "width 10, round robin over buckets) on the same kernels (lstm workload only)")
     p.add_argument("--bucket-width", type=int, default=10)
-    p.add_argument("--lengths", default="wmt", choices=["wmt", "fixed24", "clip50", "clip100"],
-                   help="LSTM request lengths: WMT-like (configs[1]) or Fig. 11's variants (L643-L681)")
+    p.add_argument("--lengths", default="wmt", choices=["wmt", "fixed24", "clip50", "clip100", "identical"],
+                   help="LSTM request lengths: WMT-like (configs[1]) or Fig. 11's variants (L643-L681); "
+                        "tree: 'identical' = every request the complete 16-leaf tree (Fig. 15, L857)")
     p.add_argument("--workers", type=int, default=1,
                    help="Algorithm 1 workers per GPU (one stream each, subgraph pinning, §8f N2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -113,7 +114,7 @@ def make_trace(wl, n, rate, seed):
         return gen.chain_trace(n, WL[wl]["vocab"], seed, rate=rate, lengths=lengths)
     if wl == "seq2seq":
         return gen.seq2seq_trace(n, WL[wl]["vocab"], seed, rate=rate)
-    return gen.tree_trace(n, WL[wl]["vocab"], seed, rate=rate)
+    return gen.tree_trace(n, WL[wl]["vocab"], seed, rate=rate, identical=LENGTHS == "identical")
 
 
 def make_weights(wl):
@@ -324,7 +325,8 @@ def reference_arm(a):
 def main():
     global LENGTHS
     a = parse()
-    LENGTHS = a.lengths if a.workload == "lstm" else "wmt"
+    LENGTHS = a.lengths if (a.workload == "lstm" and a.lengths != "identical") or \
+        (a.workload == "tree" and a.lengths == "identical") else "wmt"
     if a.impl == "reference":
         return reference_arm(a)
     import torch
@@ -537,6 +539,31 @@ def main():
         b_req = b / (24 * t_step) * world
         bound = {"t_step_b512_us": t_step * 1e6, "bound_req_s": b_req, "fraction_of_bound": value / b_req,
                  "paper": "BatchMaker at ~87% of 27,136 req/s on V100 (L679-L681)"}
+    if wl == "tree" and LENGTHS == "identical":
+        # Fig. 15 (L857): identical complete 16-leaf trees against a hard-coded ideal that packs
+        # every level of 64/16 = 4 trees into full tasks: per tree 16 leaf rows + 15 internal
+        # rows, i.e. 16/64 of a 64-row leaf task + 15/64 of a 64-row internal task
+        rng = np.random.default_rng(5)
+        b = 64
+        slots = rng.choice(1 << 16, size=3 * b, replace=False).astype(np.int32)
+        leaf_rows = np.stack([rng.integers(3, WL[wl]["vocab"], size=b), np.zeros(b), slots[:b], np.zeros(b)], 1)
+        int_rows = np.stack([slots[b:2 * b], slots[2 * b:], slots[:b], np.zeros(b)], 1)
+        lf, it = cells[gen.TREE]
+        t = {}
+        for name, cid, rows in (("leaf", lf, leaf_rows), ("internal", it, int_rows)):
+            for _ in range(5):
+                e.cell_step(cid, rows, sync=False)
+            torch.cuda.synchronize()
+            ev0.record(stream)
+            for _ in range(50):
+                e.cell_step(cid, rows, sync=False)
+            ev1.record(stream)
+            ev1.synchronize()
+            t[name] = ev0.elapsed_time(ev1) / 50 / 1e3
+        ideal = world / (16 / b * t["leaf"] + 15 / b * t["internal"])
+        bound = {"t_leaf_b64_us": t["leaf"] * 1e6, "t_internal_b64_us": t["internal"] * 1e6,
+                 "ideal_req_s": ideal, "fraction_of_ideal": value / ideal,
+                 "paper": "BatchMaker peak ~30% below the hard-coded ideal (L857)"}
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         cpu = cpu_oracle(wl, a.cpu_seconds)
@@ -545,7 +572,8 @@ def main():
                 "warmup": a.warmup, "ms_per_step": t_max * 1e3 / a.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
                 "config": {"workload": WL[wl]["config"] if LENGTHS == "wmt" else
-                           WL[wl]["config"].replace("WMT-like lengths", f"Fig. 11 lengths '{LENGTHS}'"),
+                           (WL[wl]["config"].replace("WMT-like lengths", f"Fig. 11 lengths '{LENGTHS}'")
+                            if wl == "lstm" else WL[wl]["config"] + "; identical complete 16-leaf trees (Fig. 15)"),
                            "requests_per_step": n_req,
                            "offered_rate_per_gpu": lam_star, "p90_bound_ms": bound_ms,
                            "p90_bound_kind": bound_kind,
@@ -562,7 +590,7 @@ def main():
                 # computation = first node -> completion
                 "latency_split_ms": {k: dict(zip(("p50", "p90", "p99"), (x * 1e3 for x in shard.percentiles(v))))
                                      for k, v in (("queueing", q_lat), ("computation", c_lat))},
-                "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu, "fixed_length_bound": bound,
+                "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu, "analytic_bound": bound,
                 "clocks": clk.summary(), "gpu_launches": int(st["kernel_launches"]),
                 "sched_ns_per_task": st["sched_ns"] / max(1, st["tasks"])}
         s = json.dumps(line)
