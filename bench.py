@@ -74,6 +74,8 @@ def parse():
     p.add_argument("--lengths", default="wmt", choices=["wmt", "fixed24", "clip50", "clip100", "identical"],
                    help="LSTM request lengths: WMT-like (configs[1]) or Fig. 11's variants (L643-L681); "
                         "tree: 'identical' = every request the complete 16-leaf tree (Fig. 15, L857)")
+    p.add_argument("--enc-bmax", type=int, default=512,
+                   help="Seq2Seq encoder bmax (decoder 256): 512 = BatchMaker-512,256, 256 = -256,256 (L717)")
     p.add_argument("--workers", type=int, default=1,
                    help="Algorithm 1 workers per GPU (one stream each, subgraph pinning, §8f N2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -96,6 +98,7 @@ WL = {
 }
 
 
+ENC_BMAX = 512    # --enc-bmax (Seq2Seq encoder bmax; L717: BatchMaker-512,256 vs -256,256)
 LENGTHS = "wmt"   # --lengths (LSTM): wmt | fixed24 | clip50 | clip100 (Fig. 11)
 
 
@@ -156,7 +159,7 @@ def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, kee
         cells = {gen.CHAIN: (cid, 0)}
     elif wl == "seq2seq":
         enc, dec = w["enc"], w["dec"]
-        ce = e.load_cell(bm.CELL_LSTM, L, V, 512, 0, enc.W, enc.b, enc.E)
+        ce = e.load_cell(bm.CELL_LSTM, L, V, ENC_BMAX, 0, enc.W, enc.b, enc.E)
         cd = e.load_cell(bm.CELL_LSTM_PROJ, L, V, 256, 1, dec.W, dec.b, dec.E, dec.W_out, dec.b_out)
         cells = {gen.SEQ2SEQ: (ce, cd)}
     else:
@@ -323,8 +326,9 @@ def reference_arm(a):
 
 # ------------------------------------------------------------------------------ main arm
 def main():
-    global LENGTHS
+    global LENGTHS, ENC_BMAX
     a = parse()
+    ENC_BMAX = a.enc_bmax
     LENGTHS = a.lengths if (a.workload == "lstm" and a.lengths != "identical") or \
         (a.workload == "tree" and a.lengths == "identical") else "wmt"
     if a.impl == "reference":
@@ -582,6 +586,8 @@ def main():
                            "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
                                  "step (serving)", "parallelism": f"request-sharded x{world}",
                            "persistent_kernel": bool(a.persistent), "workers_per_gpu": a.workers,
+                           "bmax": ({"encoder": ENC_BMAX, "decoder": 256} if wl == "seq2seq" else
+                                    (512 if wl == "lstm" else 64)),
                            "policy": ("cellular batching (Algorithm 1)" if policy == bm.POLICY_CELLULAR else
                                       f"graph-batching baseline: padding + bucketing, width {a.bucket_width}, "
                                       "round robin over buckets (L427)")},
