@@ -265,7 +265,7 @@ __global__ void __launch_bounds__(kThreads, 2)
   const int xkb = p.xkb > 0 ? p.xkb : 1;
   const int nst = nk / xkb;
   // wcpa (LSTM): the stage also carries the weight K blocks (loaded by the producers)
-  const bool wcpa = EPI == EPI_LSTM && p.wcpa != 0;
+  const bool wcpa = (EPI == EPI_LSTM || EPI == EPI_PROJ) && p.wcpa != 0;
   const int wblk_ = (EPI == EPI_PROJ ? 128 : G * U) * 128;
   const int kStages = wcpa ? max(2, min(kMaxStages, p.xring / ((npad * 128 + wblk_) * xkb)))
                     : p.max_stages > 0 ? min(p.max_stages, x_stages_for(npad * xkb, p.xring))
@@ -494,20 +494,25 @@ __global__ void __launch_bounds__(kThreads, 2)
     // ============================================================ projection + argmax (A10)
     float* P = reinterpret_cast<float*>(smem);  // [col][129]: reuses the drained stage ring
     constexpr int pitch = 129;
+    // p.pchunk > 0: the logits tile goes through shared memory pchunk columns at a time (a
+    // smaller footprint lets two CTAs share an SM, so all vocab tiles run in one wave)
+    const int PC = p.pchunk > 0 ? min(p.pchunk, npad) : npad;
+    const int v0 = blockIdx.y * 128;
+    for (int cc0 = 0; cc0 < npad; cc0 += PC) {
+    if (cc0 > 0) __syncthreads();  // the previous chunk's column scans are done
     if (warp < 8) {
-      for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
+      for (int c0 = cc0 + (warp >> 2) * 32; c0 < cc0 + PC && c0 < npad; c0 += 64) {
         float v[32];
         tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
 #pragma unroll
         for (int i = 0; i < 32; ++i)
-          if (c0 + i < npad) P[(c0 + i) * pitch + trow] = v[i];
+          if (c0 + i < npad) P[(c0 - cc0 + i) * pitch + trow] = v[i];
       }
     }
     tc_fence_before();
     __syncthreads();
-    if (tid == 0) phase_mark(p, 3);
-    const int v0 = blockIdx.y * 128;
-    for (int c = tid; c < ncols; c += kThreads) {
+    if (tid == 0 && cc0 == 0) phase_mark(p, 3);
+    for (int c = cc0 + tid; c < min(ncols, cc0 + PC); c += kThreads) {
       const RowDesc r = rtab[c];
       float best = -INFINITY;
       int besti = 0;
@@ -518,7 +523,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + step) * p.V + v0;
       }
       for (int i = 0; i < 128; ++i) {
-        const float z = P[c * pitch + i] + p.bias[v0 + i];
+        const float z = P[(c - cc0) * pitch + i] + p.bias[v0 + i];
         if (lg != nullptr) lg[i] = z;
         if (z > best) {  // strict: keeps the lowest index among equal maxima
           best = z;
@@ -531,6 +536,7 @@ __global__ void __launch_bounds__(kThreads, 2)
           (static_cast<unsigned long long>(ob) << 32) | (0xFFFFFFFFu - static_cast<uint32_t>(v0 + besti));
       atomicMax(p.amax + col0 + c, key);
     }
+    }  // column chunks
     __threadfence();
     __syncthreads();
     if (tid == 0) {
@@ -802,6 +808,15 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
     a.xkb = npad <= 64 ? 4 : 2;
     if (env_xkb > 0) a.xkb = env_xkb;
   }
+  // projection (BM_PROJ_SMALL, default on): cp.async weights in <= 107 KB of stages and the
+  // logits tile through shared memory 128 columns at a time, so two CTAs share an SM and all
+  // V/128 vocab tiles run in one wave instead of two
+  static const int env_proj_small = getenv("BM_PROJ_SMALL") ? atoi(getenv("BM_PROJ_SMALL")) : 1;
+  const bool proj_small = EPI == EPI_PROJ && env_proj_small && env_wcb == 0;
+  if (proj_small) {
+    a.wcpa = 1;
+    a.xkb = 1;
+  }
   const int nk_all = a.kslice / kBK;
   if (EPI == EPI_PROJ) {
     if (a.xkb > 1 && (a.H / kBK) % a.xkb != 0) a.xkb = 1;
@@ -817,9 +832,10 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   const int cbuf_bytes = (EPI == EPI_LSTM || EPI == EPI_INTERNAL) && a.pchunk == 0
                              ? (((cols + S - 1) / S) * (EPI == EPI_INTERNAL ? 2 : 1) * a.U * 4 + 1023) & ~1023
                              : 0;
+  if (proj_small) a.pchunk = npad > 128 ? 128 : 0;
   if (a.wcpa) {
     const int stage = (npad * 128 + wblk) * a.xkb;
-    const int budget = 227 * 1024 - 1024 - kTailBytes - cbuf_bytes;
+    const int budget = (proj_small ? 113 * 1024 : 227 * 1024) - 1024 - kTailBytes - cbuf_bytes;
     const int stages = std::min(kMaxStages, budget / stage);
     if (stages < 2) {
       a.wcpa = 0;  // does not fit: keep the TMA ring plan computed above
