@@ -791,6 +791,11 @@ bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w,
   }
   const int K = c.K0 + c.K1;
   c.S = std::max(1, K / 512);          // fixed K slice of 512 -> batch-invariant reduction order
+  // leaf cells (K = h): 256-wide slices (S = 4) so h/U x S = 128 CTAs stream the weights
+  // instead of 64 (BM_LEAF_S=2 keeps the 512-wide slices)
+  static const int env_leaf_s = getenv("BM_LEAF_S") ? atoi(getenv("BM_LEAF_S")) : 4;
+  if (c.epi == EPI_LEAF && env_leaf_s == 4 && e.cfg.precision == BM_PREC_BF16 && K % 1024 == 0)
+    c.S = std::min(4, K / 256);
   c.kslice = K / c.S;
   if (c.S > 8 || c.kslice % 64 != 0) return BM_E_INVAL;
   if (w->W == nullptr || w->b == nullptr) return BM_E_INVAL;

@@ -191,3 +191,28 @@ def test_batch_invariance_pair_regime(b_small, b_big):
                                  c0[i].astype(np.float64))
         assert np.max(np.abs(big_h[i] - hs)) <= STEP_TOL[bm.PREC_BF16]
         assert np.max(np.abs(big_c[i] - cs)) <= STEP_TOL[bm.PREC_BF16]
+
+
+@pytest.mark.parametrize("b_small,b_big", [(1, 64), (37, 256)])
+def test_leaf_batch_invariance(b_small, b_big):
+    """P10 for the TreeLSTM leaf cell (256-wide K slices, S = 4, tasks of <= 256 rows): a leaf's
+    result is bitwise identical in a task of b_small and of b_big rows, and within tolerance of
+    the oracle."""
+    rng = np.random.default_rng(13)
+    h, V = 1024, 300
+    e, (leaf, intern), w = tree_engine(h, V, bm.PREC_BF16, bmax=512, max_slots=2048, max_requests=2048)
+    slots = _slots(rng, b_big, 2048)
+    toks = rng.integers(3, V, size=b_big)
+    flags = bm.ROW_LAST | (np.arange(b_big) << 8)
+    rows = np.stack([toks, np.zeros(b_big), slots, flags], 1)
+    e.cell_step(leaf, rows)
+    big_h, big_c = e.result_rows(np.arange(b_big))
+    sel = np.arange(b_small)[::-1]
+    e.cell_step(leaf, rows[sel])
+    small_h, small_c = e.result_rows(np.arange(b_big)[sel])
+    assert np.array_equal(small_h, big_h[sel])
+    assert np.array_equal(small_c, big_c[sel])
+    for i in (0, b_small - 1, b_big - 1):
+        eh, ec = cells.tree_leaf(w.W_leaf, w.b_leaf, w.E[toks[i]])
+        assert np.max(np.abs(big_h[i, 0] - eh)) <= STEP_TOL[bm.PREC_BF16]
+        assert np.max(np.abs(big_c[i, 0] - ec)) <= STEP_TOL[bm.PREC_BF16]
