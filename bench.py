@@ -186,11 +186,13 @@ def pct(a, q):
     return float(np.percentile(a, q)) if len(a) else float("nan")
 
 
-def load_traffic():
-    """roofline.traffic: per-launch DRAM bytes of the LSTM cell-step kernels from the newest
-    committed ncu summary (profiles/round*/traffic_*.json, tools/traffic_from_ncu.py)."""
+def load_traffic(wl="lstm"):
+    """roofline.traffic: per-launch DRAM bytes of the workload's cell-step kernels from the newest
+    committed ncu summary (LSTM: profiles/round*/traffic_r*.json, tools/traffic_from_ncu.py;
+    seq2seq / tree: profiles/round*/traffic_<wl>_*.json, tools/traffic_wl.py)."""
     import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "round*", "traffic_*.json")))
+    pat = "traffic_r*.json" if wl == "lstm" else f"traffic_{wl}_*.json"
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "round*", pat)))
     if not files:
         return None
     d = json.load(open(files[-1]))
@@ -503,7 +505,7 @@ def main():
     achieved = st["timed_bytes"] / (t_kern / 1e3) / 1e9 if t_kern > 0 else 0.0
     tflops = st["timed_flops"] / (t_kern / 1e3) / 1e12 if t_kern > 0 else 0.0
     bf16_peak = peaks.get("bf16_tflops", 1590.0)
-    traffic = load_traffic() if wl == "lstm" and not a.persistent else None
+    traffic = load_traffic(wl) if not a.persistent else None
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
             "traffic": traffic["dram_bytes_per_launch"] if traffic else None,
             "traffic_unit": "bytes/launch (DRAM read+write, ncu, cold L2)",
