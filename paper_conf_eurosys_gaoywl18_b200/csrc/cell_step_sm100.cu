@@ -797,6 +797,10 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
     else if (small) a.xring = 32 * 1024;
     else if (env_wcb == 0) a.xkb = 2, a.wcb = 2, a.xring = 2 * 2 * npad * 128;  // 64 KB weight ring
   }
+  // internal cells up to 32 rows: 2 K blocks per hand-off still leave 3 stages in the 24 KB
+  // ring (span 15.3 -> 13.6 us at b = 1, 16.4 -> 14.8 at b = 32; at 64 rows the 2-stage
+  // minimum would overflow the two-CTAs-per-SM budget: profiles/round1/internal_plans_r1l.txt)
+  if (internal && npad <= 32 && env_wcb == 0 && env_xring == 0) a.xkb = 2;
   if (env_xkb > 0) a.xkb = env_xkb;
   // BM_WCPA=1: LSTM weights by cp.async inside the activation stages (as the CTA-pair kernel),
   // stages of xkb K blocks of (activations + 16 KB weights). Off by default here: this kernel's
