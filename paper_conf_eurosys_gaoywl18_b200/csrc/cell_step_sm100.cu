@@ -801,6 +801,13 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
   // ring (span 15.3 -> 13.6 us at b = 1, 16.4 -> 14.8 at b = 32; at 64 rows the 2-stage
   // minimum would overflow the two-CTAs-per-SM budget: profiles/round1/internal_plans_r1l.txt)
   if (internal && npad <= 32 && env_wcb == 0 && env_xring == 0) a.xkb = 2;
+  // leaf cells (256-wide K slice = 4 K blocks): the whole slice's activations in one hand-off up
+  // to 64 rows, two up to 128 (span -8% at b <= 64, -5% at 128:
+  // profiles/round1/leaf_plans_r1o.txt); a two-stage ring next to the 96 KB weight ring
+  if (EPI == EPI_LEAF && npad <= 128 && env_wcb == 0 && env_xring == 0) {
+    a.xkb = npad <= 64 ? 4 : 2;
+    a.xring = 2 * a.xkb * npad * 128;
+  }
   if (env_xkb > 0) a.xkb = env_xkb;
   // BM_WCPA=1: LSTM weights by cp.async inside the activation stages (as the CTA-pair kernel),
   // stages of xkb K blocks of (activations + 16 KB weights). Off by default here: this kernel's
