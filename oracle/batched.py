@@ -81,3 +81,47 @@ def run_tree_schedule(w, trees: Sequence[Tuple[Sequence[int], Sequence[int], Seq
         for j, (t, v) in enumerate(rows):
             st[(t, v)] = (Hn[j], C[j])
     return {t: st[(t, len(trees[t][1]) - 1)] for t in range(len(trees))}
+
+
+def run_seq2seq_forced_lockstep(enc, dec, srcs: Sequence[Sequence[int]],
+                                forced: Sequence[Sequence[int]], chunk: int = 1024):
+    """Seq2Seq in forced-token mode (decoding per L713-L715) for many requests at
+    once, in lockstep: encoder step k batches every request with > k source tokens; decoder
+    step s batches every request with > s decode steps and feeds <go> at s = 0, else the given
+    token forced[r][s-1]. Exactly the rows-concatenation of cells.seq2seq(..., forced_tokens)
+    (pinned against it in tests/test_oracle_batching.py).
+
+    Returns (h, c, sel, best): h, c = per request lists of per-layer final states; sel[r][s] =
+    logit of the forced (emitted) token forced[r][s] at step s, best[r][s] = max logit there
+    (for the argmax-validity check; the full logits are not kept)."""
+    from .cells import GO
+    n, Hd, L = len(srcs), enc.hidden, enc.layers
+    h = [np.zeros((n, Hd)) for _ in range(L)]
+    c = [np.zeros((n, Hd)) for _ in range(L)]
+
+    def stack_step(w, rows, X):
+        for l in range(L):
+            Hn, Cn = _lstm_rows(w.W[l], w.b[l], X, h[l][rows], c[l][rows])
+            h[l][rows], c[l][rows] = Hn, Cn
+            X = Hn
+        return X
+
+    S = np.array([len(s) for s in srcs])
+    for k in range(int(S.max())):
+        rows = np.flatnonzero(S > k)
+        stack_step(enc, rows, np.stack([f64(enc.E[int(srcs[r][k])]) for r in rows]))
+    T = np.array([len(f) for f in forced])
+    sel = [np.zeros(t) for t in T]
+    best = [np.zeros(t) for t in T]
+    Wo, bo = f64(dec.W_out), f64(dec.b_out)
+    for s in range(int(T.max())):
+        rows = np.flatnonzero(T > s)
+        toks = [GO if s == 0 else int(forced[r][s - 1]) for r in rows]
+        top = stack_step(dec, rows, np.stack([f64(dec.E[t]) for t in toks]))
+        for a in range(0, len(rows), chunk):
+            Z = top[a:a + chunk] @ Wo.T + bo
+            for j, r in enumerate(rows[a:a + chunk]):
+                sel[r][s] = Z[j, int(forced[r][s])]
+                best[r][s] = Z[j].max()
+    return ([[h[l][r] for l in range(L)] for r in range(n)],
+            [[c[l][r] for l in range(L)] for r in range(n)], sel, best)

@@ -24,10 +24,10 @@ Readings where the paper is silent (listed in DESIGN.md):
       within a subgraph in ascending (height, post-order index)
   S19 "idle" = outstanding tasks <= k (k = 0 is the paper's idle)
   S20 intra-subgraph successors ready at submit; inter-subgraph at retire
-  S21 same-tick order: retire (FIFO) -> admit arrivals -> Schedule if idle; every task
-      takes one tick on the single worker. Admission is FIFO in submission order: a request
-      is admitted once its arrival time has passed and every earlier-submitted request has
-      been admitted (identical to "all due arrivals in trace order" for sorted traces).
+  S21 same-tick order: retire (FIFO) -> admit every arrival due by then, in trace order ->
+      Schedule if idle; every task takes one tick on the single worker. A request is
+      admitted at its own arrival ("When a new request arrives, the request processor runs
+      the user-code to unfold the recursion", L323), independently of other requests.
   S22 slots: lowest free index. A request takes all the slots it will ever need when its
       first node is scheduled: chain/seq2seq one slot (all layers, encoder and decoder
       share it), trees one slot per node (assigned in post-order index order). All are
@@ -393,8 +393,9 @@ class Replay:
                 if not due:
                     break
                 self.retire(self.inflight_w[min(due)[1]].popleft())
-            while pending and requests[pending[0]]["arrival"] <= t:
-                i = pending.pop(0)
+            due = [i for i in pending if requests[i]["arrival"] <= t]   # S21, L323
+            pending = [i for i in pending if requests[i]["arrival"] > t]
+            for i in due:
                 q = requests[i]
                 rid_of[i] = self.admit(q["kind"], q["cells"], q.get("length", 0),
                                        q.get("decode_len", 0), q.get("left"), q.get("right"),
@@ -408,7 +409,7 @@ class Replay:
                         self.inflight_w[w].append(task)
             cand = [q[0].finish for q in self.inflight_w if q]
             if pending:
-                cand.append(requests[pending[0]]["arrival"])
+                cand.append(min(requests[i]["arrival"] for i in pending))
             if not cand:
                 break
             nt = min(cand)
@@ -524,8 +525,9 @@ class GraphBatchingReplay:
             self.now = t
             while self.inflight and self.inflight[0].finish <= t:
                 self.retire(self.inflight.popleft())
-            while pending and requests[pending[0]]["arrival"] <= t:
-                i = pending.pop(0)
+            due = [i for i in pending if requests[i]["arrival"] <= t]   # S21, L323
+            pending = [i for i in pending if requests[i]["arrival"] > t]
+            for i in due:
                 self.admit(requests[i]["length"])
             if len(self.inflight) <= self.k:
                 for task in self.schedule():
@@ -537,7 +539,7 @@ class GraphBatchingReplay:
             if self.inflight:
                 cand.append(self.inflight[0].finish)
             if pending:
-                cand.append(requests[pending[0]]["arrival"])
+                cand.append(min(requests[i]["arrival"] for i in pending))
             if not cand:
                 break
             nt = min(cand)

@@ -213,3 +213,30 @@ def test_multi_worker_traces_bit_exact(seed, n, bmax, prio, max_tasks, k, slots,
     rp = Replay(list(zip(bmax, prio)), max_slots=slots, max_tasks_to_submit=max_tasks,
                 schedule_when_outstanding_leq=k, workers=workers).run(reqs)
     _compare(e, rp)
+
+
+def test_submit_rejects_arrival_before_pending():
+    """Reading S21 / L323: each request is admitted at its own arrival. The boundary takes an
+    arrival stream: a request may not arrive before one still pending (BM_E_INVAL), so the
+    engine's FIFO admission is exactly "every due arrival, in trace order"."""
+    e, (cid,) = _engine([(bm.CELL_LSTM, 4, 0)], max_slots=64, max_requests=64)
+    e.submit(bm.REQ_CHAIN, cid, 0, [3, 3], 2.0)
+    with pytest.raises(bm.BMError):
+        e.submit(bm.REQ_CHAIN, cid, 0, [3], 1.0)
+    e.submit(bm.REQ_CHAIN, cid, 0, [3], 2.0)   # equal arrival: fine
+    e.run()
+    assert len(e.poll()) == 2
+    e.submit(bm.REQ_CHAIN, cid, 0, [3], 0.0)   # nothing pending any more: any arrival
+    e.run()
+    assert len(e.poll()) == 1
+
+
+def test_replay_admits_due_arrivals_in_trace_order():
+    """The replay admits every request whose arrival has passed, in trace order, whatever the
+    order of later entries (L323): a late-listed early arrival is not held back behind an
+    earlier-listed late one."""
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": 3.0, "length": 1},
+            {"kind": CHAIN, "cells": [0], "arrival": 0.0, "length": 1}]
+    rp = Replay([(4, 0)], max_slots=8).run(reqs)
+    assert rp.tasks[0].tick == 0.0 and len(rp.tasks[0].rows) == 1
+    assert sorted(t for _, t in rp.completions) == [1.0, 4.0]

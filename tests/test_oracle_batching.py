@@ -118,3 +118,25 @@ def test_p4_batched_executor_rejects_dependency_violation():
     w = gen.lstm_stack_weights(4, 1, 10, seed=0, bf16=False)
     with pytest.raises(AssertionError):
         batched.run_chain_schedule(w, [[3, 4]], [[(0, 1)]])
+
+
+def test_seq2seq_forced_lockstep_equals_unbatched():
+    """oracle.batched.run_seq2seq_forced_lockstep (the full-size Seq2Seq parity check's
+    executor) = cells.seq2seq(..., forced_tokens) row by row: final per-layer (h, c) to 1e-12,
+    the forced token's logit and the step maximum equal to the unbatched logits. Ragged source
+    and decode lengths, forced tokens that differ from the oracle's own argmax."""
+    h, L, V = 16, 3, 40
+    enc = gen.lstm_stack_weights(h, L, V, 31, bf16=False)
+    dec = gen.lstm_stack_weights(h, L, V, 32, projection=True, bf16=False)
+    rng = np.random.default_rng(5)
+    srcs = [list(rng.integers(3, V, size=n)) for n in (1, 4, 2, 6, 3)]
+    forced = [list(rng.integers(0, V, size=t)) for t in (3, 1, 5, 2, 4)]
+    H_, C_, sel, best = batched.run_seq2seq_forced_lockstep(enc, dec, srcs, forced, chunk=2)
+    for r in range(len(srcs)):
+        o = cells.seq2seq(enc, dec, srcs[r], len(forced[r]), forced_tokens=forced[r])
+        for l in range(L):
+            np.testing.assert_allclose(H_[r][l], o["h"][l], rtol=0, atol=1e-12)
+            np.testing.assert_allclose(C_[r][l], o["c"][l], rtol=0, atol=1e-12)
+        for s, y in enumerate(forced[r]):
+            assert abs(sel[r][s] - o["logits"][s][y]) <= 1e-12
+            assert abs(best[r][s] - o["logits"][s].max()) <= 1e-12

@@ -134,6 +134,71 @@ def test_seq2seq_forced_tokens_follow_given_sequence():
     np.testing.assert_array_equal(out["logits"][0], free["logits"][0])
 
 
+def _torch_decode_forced(enc, dec, src, fed):
+    """Independent decoder (P2 library routine): encoder = nn.LSTM over E_src; decoder step s
+    = nn.LSTM stepped on E_tgt[<go>] at s = 0 and on E_tgt[fed[s-1]] after (feed-previous
+    with the given tokens, L713-L715); logits = F.linear(h_L, W_out, b_out)."""
+    me, md = _torch_stack(enc), _torch_stack(dec)
+    Wo = torch.from_numpy(dec.W_out.astype(np.float64))
+    bo = torch.from_numpy(dec.b_out.astype(np.float64))
+    out = []
+    with torch.no_grad():
+        _, (hn, cn) = me(torch.from_numpy(enc.E[src].astype(np.float64))[:, None, :])
+        prev = gen.GO
+        for s in range(len(fed)):
+            y, (hn, cn) = md(torch.from_numpy(dec.E[prev].astype(np.float64))[None, None, :], (hn, cn))
+            out.append(torch.nn.functional.linear(y[0, 0], Wo, bo).numpy())
+            prev = int(fed[s])
+    return np.array(out), hn, cn
+
+
+@pytest.mark.parametrize("k", [0, 2, 4])
+def test_p2_seq2seq_forced_token_mode_vs_torch(k):
+    """Forced-token mode (decoding per L715) pinned against an independent decoder:
+    take the free run's tokens and change the one emitted at step k. Then (i) the logits of
+    steps <= k are exactly the free run's (the change only reaches the input of step k+1),
+    (ii) every step's logits and the final per-layer (h, c) equal torch nn.LSTM stepped on the
+    forced tokens, and (iii) step k+1 differs from the free run (the forced token was fed,
+    not the oracle's own argmax). A decoder that feeds its own argmax fails (ii)."""
+    h, L, V, T = 16, 4, 50, 6
+    enc = _w(h, L, V, seed=20)
+    dec = _w(h, L, V, seed=21, projection=True)
+    src = [9, 31, 4, 17, 40]
+    free = cells.seq2seq(enc, dec, src, T)
+    forced = list(free["tokens"])
+    forced[k] = (forced[k] + 7) % V
+    out = cells.seq2seq(enc, dec, src, T, forced_tokens=forced)
+    np.testing.assert_array_equal(out["logits"][:k + 1], free["logits"][:k + 1])
+    ref, hn, cn = _torch_decode_forced(enc, dec, src, forced)
+    np.testing.assert_allclose(out["logits"], ref, rtol=0, atol=1e-13)
+    for l in range(L):
+        np.testing.assert_allclose(out["h"][l], hn[l, 0].numpy(), rtol=0, atol=1e-14)
+        np.testing.assert_allclose(out["c"][l], cn[l, 0].numpy(), rtol=0, atol=1e-14)
+    assert np.max(np.abs(out["logits"][k + 1] - free["logits"][k + 1])) > 1e-6
+    # the oracle's own argmax is still reported for the validity check
+    assert out["tokens"] == [cells.argmax_lowest(z) for z in out["logits"]]
+
+
+def test_seq2seq_forced_tokens_terminate_at_forced_eos():
+    """With eos_stop, termination follows the FED token (N1 under forced-token mode): forcing
+    the eos id at step k ends decoding after step k; the state then equals torch's after k+1
+    steps."""
+    h, L, V, T, k = 16, 2, 40, 8, 3
+    enc = _w(h, L, V, seed=22)
+    dec = _w(h, L, V, seed=23, projection=True)
+    src = [5, 6, 7]
+    free = cells.seq2seq(enc, dec, src, T)
+    eos = (free["tokens"][k] + 1) % V
+    forced = [t if t != eos else (t + 2) % V for t in free["tokens"]]
+    forced[k] = eos
+    out = cells.seq2seq(enc, dec, src, T, forced_tokens=forced, eos_id=eos)
+    assert len(out["logits"]) == k + 1 and out["fed_tokens"][-1] == eos
+    ref, hn, cn = _torch_decode_forced(enc, dec, src, forced[:k + 1])
+    np.testing.assert_allclose(out["logits"], ref, rtol=0, atol=1e-13)
+    for l in range(L):
+        np.testing.assert_allclose(out["h"][l], hn[l, 0].numpy(), rtol=0, atol=1e-14)
+
+
 # ----------------------------------------------------------------------------- P3 (trees)
 def _tree_w(h=8, V=16, seed=0):
     return gen.tree_weights(h, V, seed, bf16=False)
