@@ -3,30 +3,49 @@
 
 Workload (BASELINE.json configs[1], the metric's configuration): 1-layer LSTM, h = 1024,
 WMT-like sentence lengths (mean 24, max 330; L421, L635), Poisson open-loop arrivals (L423),
-bmax 512 (L429), MaxTasksToSubmit 5 (L379), synthetic seeded weights/tokens.
-`--workload seq2seq|tree` runs configs[2] / configs[3] instead.
+bmax 512 (L429), MaxTasksToSubmit 5 (L379), synthetic seeded weights/tokens. The default run
+also measures configs[2] (Seq2Seq) and configs[3] (TreeLSTM) with the same protocol and
+reports them under "extra_workloads" (--extra none skips them); `--workload seq2seq|tree`
+makes one of them the headline instead.
 
-A STEP = one open-loop Poisson trace of --reqs requests at the offered rate lambda* pushed
-through the whole hot path (A1 unfold at admission, A2-A3 Algorithm 1, A4 slot pool, A5 launch,
-A6-A9 fused gather/tcgen05/gate/scatter kernels, A12 completion signal, A13 poll/retire),
-by the C-ABI engine's own event loop (bm_run). lambda* = the highest rate of a load sweep
-(run first, untimed) whose p90 latency stays within the bound (--p90-ms, default 12 ms: the
-paper's flat-region LSTM p90, L489).
+Protocol (L423 "adjust the average inter-arrival time", L489 p90 vs throughput):
+  1. saturation estimate mu: a burst trace (every request arrives at t = 0);
+  2. sustained load sweep, untimed: offered rate lambda on a grid of fractions of mu, each point
+     an open-loop Poisson trace of >= 100 k requests or >= 5 s; a point is SUSTAINED when the
+     achieved rate is within 2% of the offered one (no backlog growth); p50/p90/p99 per point;
+  3. lambda* = the highest sustained offered rate whose p90 is within the bound (12 ms, the
+     paper's flat-region LSTM p90, L489; Seq2Seq: the knee, 2x the lowest-load p90), refined
+     by bisection against the next (failing) grid point;
+  4. a STEP = one open-loop Poisson trace of --reqs requests at lambda* through the whole hot
+     path (A1 unfold, A2-A3 Algorithm 1, A4 slots, A5 launch, A6-A10 kernels, A12 signal, A13
+     retire) by the C-ABI engine's own event loop (bm_run); W warm-up steps, K timed steps.
 
 value    = requests completed by all ranks / max over ranks of the device time of the K steps
-e2e      = same, through the public API with host buffers: per step the bm_request arrays are
-           submitted from host memory, row descriptors (tokens inside) go host->device from
-           pinned memory on every Schedule call, and all final h rows come back device->host
-roofline = the LSTM cell-step kernel: algorithmic bytes / CUDA-event time of every launch in
-           the timed region, against MEASURED_PEAKS.json
-Multi-GPU (torchrun): one engine per GPU, requests sharded by rank (weak scaling: each rank
-runs its own lambda* Poisson stream), weights broadcast once from rank 0 with NCCL; no
-collective on the per-step path.
+           (CUDA events on the engine stream around each step; a 256 MB buffer is written
+           between steps, > the 126 MB L2)
+e2e      = same metric through the public API with host buffers: every step submits the
+           bm_request arrays from host memory, row descriptors go host->device from pinned
+           memory at every Schedule call, and every request's final h comes back device->host
+roofline = the kernel class with the most device time in the timed steps. EVERY launch is timed
+           on the device (%globaltimer span: first CTA past its dependency wait .. last CTA
+           done; include/bm.h "measurement"), and the same launches' algorithmic bytes / flops
+           are summed by the library, so time, bytes and flops cover one population. Each
+           launch is bound by the larger of bytes/HBM and flops/tensor peak (MEASURED_PEAKS.json:
+           hbm_gbs, bf16_tflops_sustained -- the kernels run inside a long step); frac_binding
+           = sum of roof times / sum of device time; bound/achieved/peak/frac = the roof that
+           dominates that sum. Per-class entries in roofline.kernels; traffic = ncu DRAM bytes
+           per launch of the class captured inside this bench workload (profiles/round*/).
+Multi-GPU: `--gpus N` re-launches itself under torch.distributed.run (one process per GPU)
+unless WORLD_SIZE is already N. One engine per GPU, requests sharded by rank (weak scaling:
+each rank runs its own lambda* Poisson stream), weights broadcast once from rank 0 with NCCL
+and adopted by bm_load_cell straight from device memory; no collective on the per-step path.
 """
 from __future__ import annotations
 
 import argparse
+import glob
 import json
+import math
 import os
 import statistics
 import subprocess
@@ -47,6 +66,9 @@ sys.path.insert(0, ROOT)
 from workloads import gen  # noqa: E402
 
 METRIC = "requests/sec at p90-latency bound"
+POINT_REQS = 100_000     # sweep point: >= 100 k requests ...
+POINT_SECONDS = 5.0      # ... or >= 5 s of offered load, whichever is reached first
+SUSTAINED = 0.98         # achieved / offered of a sustained point
 
 
 def parse():
@@ -56,7 +78,10 @@ def parse():
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="lstm", choices=["lstm", "seq2seq", "tree"])
-    p.add_argument("--reqs", type=int, default=0, help="requests per step (0 = per-workload default)")
+    p.add_argument("--extra", default="auto",
+                   help="comma list of extra workloads measured in the same run (auto: seq2seq,tree "
+                        "when the headline is lstm at N = 1; none)")
+    p.add_argument("--reqs", type=int, default=0, help="requests per timed step (0 = per-workload default)")
     p.add_argument("--p90-ms", type=float, default=0.0,
                    help="p90 bound; 0 = per-workload default (12 ms, L489; Seq2Seq: the knee, "
                         "2x the lowest-load p90, since Fig. 13's values are not legible)")
@@ -80,6 +105,10 @@ def parse():
                    help="Algorithm 1 workers per GPU (one stream each, subgraph pinning, §8f N2)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
+    p.add_argument("--quick", action="store_true", help="short sweep (development runs, profiling)")
+    p.add_argument("--dry", action="store_true",
+                   help="functional check without a GPU: BM_CLOCK_DRY engines (scheduler only, virtual "
+                        "ticks: one tick per task), gloo collectives; no kernels, so no timing claims")
     p.add_argument("--out", default="")
     return p.parse_args()
 
@@ -87,16 +116,20 @@ def parse():
 # ------------------------------------------------------------------------------ workloads
 WL = {
     "lstm": dict(config="BASELINE configs[1]: 1-layer LSTM h=1024, WMT-like lengths, Poisson arrivals, "
-                        "bmax 512, 1 B200", hidden=1024, layers=1, vocab=32768, reqs=20000,
-                 p90_ms=12.0, lookahead=2, persistent=0),
+                        "bmax 512, 1 B200", hidden=1024, layers=1, vocab=32768, reqs=100_000,
+                 p90_ms=12.0, lookahead=2, persistent=0,
+                 fracs=(0.05, 0.25, 0.5, 0.7, 0.8, 0.85, 0.9, 0.95, 1.0, 1.05)),
     "seq2seq": dict(config="BASELINE configs[2]: Seq2Seq 4+4 layer LSTM h=1024, vocab 32768, greedy "
                            "decode, encoder/decoder bmax 512/256", hidden=1024, layers=4, vocab=32768,
-                    reqs=4000, p90_ms=None, lookahead=1, persistent=0),
+                    reqs=20_000, p90_ms=None, lookahead=1, persistent=0,
+                    fracs=(0.05, 0.5, 0.7, 0.8, 0.9, 0.95, 1.0)),
     "tree": dict(config="BASELINE configs[3]: TreeLSTM h=1024, TreeBank-shaped binary trees, leaf/internal "
-                        "cells batched separately, bmax 64", hidden=1024, layers=1, vocab=32768, reqs=6000,
-                 p90_ms=12.0, lookahead=2, persistent=0),
+                        "cells batched separately, bmax 64", hidden=1024, layers=1, vocab=32768, reqs=50_000,
+                 p90_ms=12.0, lookahead=2, persistent=0,
+                 fracs=(0.05, 0.5, 0.7, 0.8, 0.9, 0.95, 1.0, 1.05)),
 }
-
+EXTRA_REQS = {"seq2seq": 20_000, "tree": 50_000}   # per timed step of an extra workload
+EXTRA_STEPS = 3
 
 ENC_BMAX = 512    # --enc-bmax (Seq2Seq encoder bmax; L717: BatchMaker-512,256 vs -256,256)
 LENGTHS = "wmt"   # --lengths (LSTM): wmt | fixed24 | clip50 | clip100 (Fig. 11)
@@ -112,12 +145,13 @@ def chain_lengths(n, seed, kind):
 
 
 def make_trace(wl, n, rate, seed):
+    lengths_kind = LENGTHS if wl in ("lstm", "tree") else "wmt"
     if wl == "lstm":
-        lengths = None if LENGTHS == "wmt" else chain_lengths(n, seed, LENGTHS)
+        lengths = None if lengths_kind in ("wmt", "identical") else chain_lengths(n, seed, lengths_kind)
         return gen.chain_trace(n, WL[wl]["vocab"], seed, rate=rate, lengths=lengths)
     if wl == "seq2seq":
         return gen.seq2seq_trace(n, WL[wl]["vocab"], seed, rate=rate)
-    return gen.tree_trace(n, WL[wl]["vocab"], seed, rate=rate, identical=LENGTHS == "identical")
+    return gen.tree_trace(n, WL[wl]["vocab"], seed, rate=rate, identical=lengths_kind == "identical")
 
 
 def make_weights(wl):
@@ -145,14 +179,32 @@ def weight_arrays(w):
     return out
 
 
+class DevWeights:
+    """Weights as device tensors (after the NCCL broadcast), same attribute names as gen's
+    dataclasses, so bm_load_cell adopts them in place (include/bm.h bm_weights)."""
+
+    def __init__(self, src, tensors, key):
+        for f in ("W", "b"):
+            if hasattr(src, f):
+                setattr(self, f, [tensors[f"{key}.{f}{i}"] for i in range(len(getattr(src, f)))])
+        for f in ("E", "W_out", "b_out", "W_leaf", "b_leaf", "U", "b_int"):
+            if getattr(src, f, None) is not None:
+                setattr(self, f, tensors[f"{key}.{f}"])
+            elif not hasattr(self, f):
+                setattr(self, f, None)
+
+
 # ------------------------------------------------------------------------------ engine
 def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, keep=0, persistent=0,
-                 policy=0, bucket_width=10, workers=1):
+                 policy=0, bucket_width=10, workers=1, peaks=None, dry=False):
     h, L, V = WL[wl]["hidden"], WL[wl]["layers"], WL[wl]["vocab"]
-    e = bm.Engine(device=device, hidden=h, pool_layers=L, max_slots=1 << 16, max_requests=max_requests,
+    peaks = peaks or {}
+    e = bm.Engine(device=device, clock=bm.CLOCK_DRY if dry else bm.CLOCK_WALL, hidden=h, pool_layers=L,
+                  max_slots=1 << 16, max_requests=max_requests,
                   schedule_when_outstanding_leq=lookahead, time_kernels=time_kernels, keep_results=keep,
                   max_decode_len=340, record_log=0, persistent=persistent, policy=policy,
-                  bucket_width=bucket_width, workers=workers)
+                  bucket_width=bucket_width, workers=workers,
+                  roof_hbm_gbs=peaks.get("hbm_gbs", 0.0), roof_tc_tflops=peaks.get("tc_tflops", 0.0))
     if wl == "lstm":
         c = w["cell"]
         cid = e.load_cell(bm.CELL_LSTM, L, V, 512, 0, c.W, c.b, c.E)
@@ -170,16 +222,18 @@ def build_engine(bm, wl, w, device, max_requests, lookahead, time_kernels=1, kee
     return e, cells
 
 
-def run_trace(e, prepared, n):
-    """Submit a prepared trace and drive it to completion; returns (wall s, latencies s)."""
+def run_trace(e, prepared, n, dry=False):
+    """Submit a prepared trace and drive it to completion; returns (duration, completions):
+    wall seconds, or (DRY) virtual ticks from the first arrival to the last completion."""
     e.submit_many(prepared)
     t0 = time.perf_counter()
     done = e.run()
     t1 = time.perf_counter()
     comp = e.poll_array(n + 16)
     assert done == n and len(comp) == n, (done, len(comp), n)
-    lat = comp["t_done"] - comp["t_arrival"]
-    return t1 - t0, lat
+    if dry:
+        return max(1.0, float(comp["t_done"].max() - comp["t_arrival"].min())), comp
+    return t1 - t0, comp
 
 
 def pct(a, q):
@@ -187,17 +241,25 @@ def pct(a, q):
 
 
 def load_traffic(wl="lstm"):
-    """roofline.traffic: per-launch DRAM bytes of the workload's cell-step kernels from the newest
-    committed ncu summary (LSTM: profiles/round*/traffic_r*.json, tools/traffic_from_ncu.py;
-    seq2seq / tree: profiles/round*/traffic_<wl>_*.json, tools/traffic_wl.py)."""
-    import glob
-    pat = "traffic_r*.json" if wl == "lstm" else f"traffic_{wl}_*.json"
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "round*", pat)))
+    """Per-class ncu DRAM bytes per launch captured inside this bench workload, newest committed
+    summary (profiles/round*/traffic_<wl>.json, tools/traffic_from_ncu.py)."""
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "round*", f"traffic_{wl}.json")))
     if not files:
         return None
     d = json.load(open(files[-1]))
     d["file"] = os.path.relpath(files[-1], ROOT)
     return d
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        pk = json.load(open(path))
+        return {"hbm_gbs": pk["hbm_gbs"], "tc_tflops": pk.get("bf16_tflops_sustained", pk["bf16_tflops"]),
+                "source": "MEASURED_PEAKS.json (hbm_gbs: measured copy; bf16_tflops_sustained: cuBLAS bf16 "
+                          "back to back for 4 s -- the kernels run inside a long step)"}
+    return {"hbm_gbs": 6650.0, "tc_tflops": 1400.0,
+            "source": "fallback of /opt/skills/guides/B200_PROFILING.md (6.65 TB/s; 1.4 PF/s sustained)"}
 
 
 # ------------------------------------------------------------------------------ clocks
@@ -280,7 +342,6 @@ def cpu_oracle(wl, seconds, seed=1000):
     import multiprocessing as mp
     cores = os.cpu_count() or 1
     trace = make_trace(wl, 20000, None, seed)
-    # calibrate the cost of one cell step on this host
     probe = [i for i in range(len(trace)) if _cost(trace[i]) >= 8][:1]
     n_est, dt = _oracle_worker((wl, probe, seed, 20000))
     per_step = dt / _cost(trace[probe[0]])
@@ -326,148 +387,253 @@ def reference_arm(a):
     print(json.dumps(line), flush=True)
 
 
-# ------------------------------------------------------------------------------ main arm
-def main():
-    global LENGTHS, ENC_BMAX
-    a = parse()
-    ENC_BMAX = a.enc_bmax
-    LENGTHS = a.lengths if (a.workload == "lstm" and a.lengths != "identical") or \
-        (a.workload == "tree" and a.lengths == "identical") else "wmt"
-    if a.impl == "reference":
-        return reference_arm(a)
-    import torch
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    # one GPU per rank (NCCL over NVLink). With fewer GPUs than ranks (a functional check of the
-    # multi-rank path on one GPU) ranks share devices and the few collectives go over gloo.
-    ndev = max(1, torch.cuda.device_count())
-    local = local_rank % ndev
-    shared = world > ndev
-    torch.cuda.set_device(local)
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
-        if shared:
-            dist.init_process_group("gloo")
-        else:
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    coll_dev = None if shared else torch.device("cuda", local)
-    from paper_conf_eurosys_gaoywl18_b200 import bm, shard
+# ------------------------------------------------------------------------------ roofline
+def roofline(bm, st, peaks, steps, traffic=None):
+    """Per kernel class: every launch of the timed steps (device spans) against the same launches'
+    algorithmic bytes / flops; the headline entry is the class with the most device time."""
+    kern = {}
+    for k in range(bm.K_CLASSES):
+        n = st["k_launches"][k]
+        if not n:
+            continue
+        span_ms = st["k_span_ms"][k]
+        nspan = st["k_span_launches"][k]
+        t_hbm, t_tc, t_bind = st["k_roof_hbm_ms"][k], st["k_roof_tc_ms"][k], st["k_roof_ms"][k]
+        tensor = t_tc >= t_hbm
+        sec = span_ms / 1e3 if span_ms > 0 else float("nan")
+        ach = (st["k_flops"][k] / sec / 1e12) if tensor else (st["k_bytes"][k] / sec / 1e9)
+        peak = peaks["tc_tflops"] if tensor else peaks["hbm_gbs"]
+        ent = {"name": bm.K_NAMES.get(k, str(k)), "launches": int(n), "timed_launches": int(nspan),
+               "rows_per_launch": st["k_rows"][k] / n, "span_us_per_launch": span_ms * 1e3 / max(1, nspan),
+               "ms_per_step": span_ms / steps,
+               "bytes_per_launch": st["k_bytes"][k] / n, "flops_per_launch": st["k_flops"][k] / n,
+               "bound": "tensor" if tensor else "hbm", "achieved": ach, "peak": peak,
+               "unit": "TFLOP/s" if tensor else "GB/s", "frac": ach / peak,
+               "achieved_GBps": st["k_bytes"][k] / sec / 1e9, "achieved_TFLOPs": st["k_flops"][k] / sec / 1e12,
+               "frac_binding": t_bind / span_ms if span_ms > 0 else None,
+               "roof_hbm_ms": t_hbm, "roof_tc_ms": t_tc, "roof_binding_ms": t_bind, "span_ms": span_ms}
+        if traffic and str(k) in traffic.get("classes", {}):
+            ent["traffic"] = traffic["classes"][str(k)]["dram_bytes_per_launch"]
+            ent["traffic_l2_to_sm"] = traffic["classes"][str(k)].get("l2_to_sm_bytes_per_launch")
+        kern[str(k)] = ent
+    if not kern:
+        return None, {}
+    total_span = sum(v["span_ms"] for v in kern.values())
+    for v in kern.values():
+        v["share_of_kernel_time"] = v["span_ms"] / total_span if total_span else None
+    top = max(kern.values(), key=lambda v: v["span_ms"])
+    roof = {"bound": top["bound"], "achieved": top["achieved"], "peak": top["peak"], "unit": top["unit"],
+            "frac": top["frac"], "traffic": top.get("traffic"), "traffic_l2_to_sm": top.get("traffic_l2_to_sm"),
+            "traffic_unit": "bytes/launch (ncu dram__bytes_read.sum + dram__bytes_write.sum, inside this bench "
+                            "workload)",
+            "traffic_source": traffic["file"] if traffic else None,
+            "kernel": top["name"], "frac_binding": top["frac_binding"],
+            "span_us_per_launch": top["span_us_per_launch"], "rows_per_launch": top["rows_per_launch"],
+            "launches": top["launches"], "timed_launches": top["timed_launches"],
+            "peak_source": peaks["source"],
+            "all_kernels_frac_binding": sum(v["roof_binding_ms"] for v in kern.values()) / total_span
+            if total_span else None,
+            "kernel_ms_per_step": total_span / steps,
+            "timing": "every launch of the timed steps, device span (%globaltimer: first CTA past its dependency "
+                      "wait .. last CTA done) accumulated per kernel class by the launch's last CTA; bytes/flops "
+                      "= the same launches' algorithmic bytes/flops (DESIGN.md §6)",
+            "kernels": kern}
+    return roof, kern
 
-    wl = a.workload
-    n_req = a.reqs or WL[wl]["reqs"]
-    if a.lookahead < 0:
-        a.lookahead = WL[wl]["lookahead"]
-    if a.persistent < 0:
-        a.persistent = WL[wl]["persistent"]
-    policy = bm.POLICY_GRAPH if a.policy == "graph" else bm.POLICY_CELLULAR
+
+# ------------------------------------------------------------------------------ one workload
+class Ctx:
+    pass
+
+
+def measure_point(ctx, e, prep, n, lam):
+    """One open-loop Poisson point at offered rate lam (unit-rate trace rescaled)."""
+    prep.set_time_scale(1.0 / lam)
+    wall, comp = run_trace(e, prep, n, ctx.dry)
+    lat = comp["t_done"] - comp["t_arrival"]
+    p50, p90, p99 = (ctx.allmax(pct(lat, q)) for q in (50, 90, 99))
+    achieved = ctx.allmin(n / wall)
+    return {"offered": lam, "achieved": achieved, "n": n, "seconds": wall, "p50_ms": p50 * 1e3,
+            "p90_ms": p90 * 1e3, "p99_ms": p99 * 1e3, "sustained": bool(achieved >= SUSTAINED * lam)}
+
+
+def run_workload(ctx, a, wl, n_req, steps, warmup, headline):
+    bm, rank, local = ctx.bm, ctx.rank, ctx.local
+    lookahead = a.lookahead if (headline and a.lookahead >= 0) else WL[wl]["lookahead"]
+    persistent = a.persistent if (headline and a.persistent >= 0) else WL[wl]["persistent"]
+    policy = bm.POLICY_GRAPH if (headline and a.policy == "graph") else bm.POLICY_CELLULAR
     if policy == bm.POLICY_GRAPH and wl != "lstm":
         raise SystemExit("--policy graph: chain LSTM workload only (reading G5)")
     if policy == bm.POLICY_GRAPH:
-        a.persistent = 0
-    # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink), never again
+        persistent = 0
+    workers = a.workers if headline else 1
+    # ---- weights: generated on rank 0, broadcast once over NCCL (NVLink) and adopted in place
     w = make_weights(wl)
-    if dist is not None:
-        shard.broadcast_arrays(weight_arrays(w), dist, device=coll_dev)
-    e, cells = build_engine(bm, wl, w, local, max_requests=max(n_req, 1 << 15) + 64, lookahead=a.lookahead,
-                            persistent=a.persistent, policy=policy, workers=a.workers, bucket_width=a.bucket_width)
-    stream = torch.cuda.ExternalStream(e.stream(), device=torch.device("cuda", local))
-
-    def barrier():
-        torch.cuda.synchronize()
-        if dist is not None:
-            dist.barrier()
-
-    def allmax(x):
-        return shard.reduce_max(x, dist, device=coll_dev)
-
-    # ---- calibrate saturation: every request of a trace arrives at t = 0
-    burst = make_trace(wl, n_req, None, seed=shard.rank_seed(7, rank))
+    if ctx.dist is not None:
+        tens = ctx.shard.broadcast_tensors(weight_arrays(w), ctx.dist, device=ctx.coll_dev)
+        if ctx.coll_dev is not None:
+            w = {k: DevWeights(v, tens, k) for k, v in w.items()}
+    sweep_n = POINT_REQS if not a.quick else 20_000
+    max_req = max(n_req, sweep_n) + 64
+    e, cells = build_engine(bm, wl, w, local, max_requests=max_req, lookahead=lookahead, persistent=persistent,
+                            policy=policy, workers=workers, bucket_width=a.bucket_width, peaks=ctx.peaks,
+                            dry=ctx.dry)
+    stream = None if ctx.dry else ctx.torch.cuda.ExternalStream(e.stream(), device=ctx.torch.device("cuda", local))
+    # ---- 1. saturation estimate: every request of a trace arrives at t = 0
+    n_burst = min(n_req, 20_000 if wl == "seq2seq" else 50_000)
+    burst = make_trace(wl, n_burst, None, seed=ctx.shard.rank_seed(7, rank))
     pb = e.prepare_requests(burst, cells)
-    run_trace(e, pb, n_req)                      # warm (also JIT of nothing: all AOT)
-    dt, _ = run_trace(e, pb, n_req)
-    mu = n_req / dt
-    # ---- load sweep (open loop), untimed: highest rate whose p90 <= bound
-    curve = []
+    run_trace(e, pb, n_burst, ctx.dry)
+    dt, _ = run_trace(e, pb, n_burst, ctx.dry)
+    mu = ctx.allmin(n_burst / dt)
+    # ---- 2./3. sustained sweep (untimed) -> lambda*
+    curve, bounds = [], None
     bound_kind = "absolute"
-    if a.rate > 0:
+    if a.rate > 0 and headline:
         lam_star = a.rate
         bound_ms = a.p90_ms or WL[wl]["p90_ms"] or 12.0
     else:
-        for frac in (0.05, 0.1, 0.2, 0.35, 0.5, 0.65, 0.8, 0.9, 1.0, 1.1):
-            lam = frac * mu
-            n_pt = int(max(2000, min(n_req, lam * 0.25)))
-            tr = make_trace(wl, n_pt, lam, seed=shard.rank_seed(100, rank))
-            p = e.prepare_requests(tr, cells)
-            wall, lat = run_trace(e, p, n_pt)
-            p50, p90, p99 = (allmax(pct(lat, q)) for q in (50, 90, 99))
-            curve.append({"offered": lam, "achieved": n_pt / wall, "p50_ms": p50 * 1e3, "p90_ms": p90 * 1e3,
-                          "p99_ms": p99 * 1e3})
-        bound_ms = a.p90_ms or WL[wl]["p90_ms"]
-        if not bound_ms:   # the knee: 2x the lowest-load p90
-            bound_ms = 2.0 * curve[0]["p90_ms"]
+        unit = make_trace(wl, sweep_n, 1.0, seed=ctx.shard.rank_seed(100, rank))   # unit-rate Poisson
+        pu = e.prepare_requests(unit, cells)
+        fracs = WL[wl]["fracs"] if not a.quick else (0.05, 0.5, 0.8, 0.95)
+        for f in fracs:
+            lam = f * mu
+            n_pt = int(min(sweep_n, max(2000, math.ceil(POINT_SECONDS * lam))))
+            pp = pu if n_pt == sweep_n else e.prepare_requests(unit[:n_pt], cells)
+            curve.append(measure_point(ctx, e, pp, n_pt, lam))
+        bound_ms = (a.p90_ms if headline else 0) or WL[wl]["p90_ms"]
+        knee_ms = 2.0 * curve[0]["p90_ms"]
+        if not bound_ms:
+            bound_ms = knee_ms
             bound_kind = "knee (2x lowest-load p90)"
 
+        def ok(c, b):
+            return c["sustained"] and c["p90_ms"] <= b
+
         def best_under(b):
-            ok = [c["offered"] for c in curve if c["p90_ms"] <= b]
-            return max(ok) if ok else None
-        lam_star = best_under(bound_ms) or curve[0]["offered"]
-        knee_ms = 2.0 * curve[0]["p90_ms"]
-        bounds = {"12ms": best_under(12.0), "knee": best_under(knee_ms), "knee_ms": knee_ms}
-    # ---- timed steps at lambda*
-    trace = make_trace(wl, n_req, lam_star, seed=shard.rank_seed(1000, rank))
+            good = [c["offered"] for c in curve if ok(c, b)]
+            return max(good) if good else None
+        # bisection between the best passing point and the next grid point above it
+        lo = best_under(bound_ms) or curve[0]["offered"]
+        above = [c["offered"] for c in curve if c["offered"] > lo]
+        hi = min(above) if above else None
+        for _ in range(2 if (hi is not None and not a.quick) else 0):
+            mid = 0.5 * (lo + hi)
+            n_pt = int(min(sweep_n, max(2000, math.ceil(POINT_SECONDS * mid))))
+            pp = pu if n_pt == sweep_n else e.prepare_requests(unit[:n_pt], cells)
+            c = measure_point(ctx, e, pp, n_pt, mid)
+            c["bisection"] = True
+            curve.append(c)
+            lo, hi = (mid, hi) if ok(c, bound_ms) else (lo, mid)
+        lam_star = lo
+        curve.sort(key=lambda c: c["offered"])
+        bounds = {"12ms": best_under(12.0), "knee": best_under(knee_ms), "knee_ms": knee_ms,
+                  "rule": f"highest offered rate with achieved >= {SUSTAINED:.0%} of offered and p90 within "
+                          "the bound; points of >= 100 k requests or >= 5 s"}
+    # ---- 4. timed steps at lambda*
+    trace = make_trace(wl, n_req, 1.0, seed=ctx.shard.rank_seed(1000, rank))
     prep = e.prepare_requests(trace, cells)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
-    for _ in range(a.warmup):
-        run_trace(e, prep, n_req)
+    prep.set_time_scale(1.0 / lam_star)
+    flush = None if ctx.dry else ctx.torch.empty(256 << 20, dtype=ctx.torch.uint8, device="cuda")  # > L2
+    for _ in range(warmup):
+        run_trace(e, prep, n_req, ctx.dry)
     e.reset_stats()
-    barrier()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ctx.barrier()
     dev_ms = 0.0
-    lats, queue, compute = [], [], []
+    lats, queue, compute, achieved = [], [], [], []
     with ClockSampler(local) as clk:
-        for _ in range(a.steps):
-            flush.zero_()
-            torch.cuda.synchronize()
-            e.submit_many(prep)
-            ev0.record(stream)
-            done = e.run()
-            ev1.record(stream)
-            ev1.synchronize()
-            assert done == n_req
-            dev_ms += ev0.elapsed_time(ev1)
-            comp = e.poll_array(n_req + 16)
+        for _ in range(steps):
+            if ctx.dry:   # virtual ticks stand in for the device time (functional check only)
+                wall, comp = run_trace(e, prep, n_req, True)
+                dev_ms += wall * 1e3
+            else:
+                ev0, ev1 = ctx.torch.cuda.Event(enable_timing=True), ctx.torch.cuda.Event(enable_timing=True)
+                flush.zero_()
+                ctx.torch.cuda.synchronize()
+                e.submit_many(prep)
+                ev0.record(stream)
+                t0 = time.perf_counter()
+                done = e.run()
+                wall = time.perf_counter() - t0
+                ev1.record(stream)
+                ev1.synchronize()
+                assert done == n_req
+                dev_ms += ev0.elapsed_time(ev1)
+                comp = e.poll_array(n_req + 16)
             lats.append(comp["t_done"] - comp["t_arrival"])
             queue.append(comp["t_first"] - comp["t_arrival"])   # E5 (Fig. 9, L597): queueing
             compute.append(comp["t_done"] - comp["t_first"])     # ... and computation time
-    barrier()
+            achieved.append(n_req / wall)
+    ctx.barrier()
     st = e.stats()
-    lat = shard.gather_samples(np.concatenate(lats), dist, device=coll_dev)
-    q_lat = shard.gather_samples(np.concatenate(queue), dist, device=coll_dev)
-    c_lat = shard.gather_samples(np.concatenate(compute), dist, device=coll_dev)
-    t_max = allmax(dev_ms / 1e3)
-    total = n_req * a.steps * world
+    launch_log = None if ctx.dry else e.launch_log()
+    lat = ctx.shard.gather_samples(np.concatenate(lats), ctx.dist, device=ctx.coll_dev)
+    q_lat = ctx.shard.gather_samples(np.concatenate(queue), ctx.dist, device=ctx.coll_dev)
+    c_lat = ctx.shard.gather_samples(np.concatenate(compute), ctx.dist, device=ctx.coll_dev)
+    t_max = ctx.allmax(dev_ms / 1e3)
+    total = n_req * steps * ctx.world
     value = total / t_max
-    p50, p90, p99 = shard.percentiles(lat)   # over the union of all ranks' requests
-    # ---- e2e: public API with host buffers (submit from host, descriptors H2D every Schedule
-    #      call inside bm_run, final h rows D2H), timed on the host clock around the whole thing
-    e2, cells2 = build_engine(bm, wl, w, local, max_requests=n_req + 64, lookahead=a.lookahead,
-                              time_kernels=0, keep=1, persistent=a.persistent, policy=policy, workers=a.workers,
-                              bucket_width=a.bucket_width)
+    p50, p90, p99 = ctx.shard.percentiles(lat)   # over the union of all ranks' requests
+    roof, kern = (None, {}) if ctx.dry else roofline(bm, st, ctx.peaks, steps,
+                                                     None if persistent else load_traffic(wl))
+    out = {"value": value, "unit": "requests/sec", "ms_per_step": t_max * 1e3 / steps,
+           "offered_rate_per_gpu": lam_star, "achieved_over_offered": float(np.mean(achieved)) / lam_star,
+           "p90_bound_ms": bound_ms, "p90_bound_kind": bound_kind, "max_offered_rate_under": bounds,
+           "saturation_burst_rate_per_gpu": mu, "lookahead_k": lookahead, "requests_per_step": n_req,
+           "latency_ms": {"p50": p50 * 1e3, "p90": p90 * 1e3, "p99": p99 * 1e3},
+           # Fig. 9's decomposition (L597): queueing = arrival -> first node scheduled,
+           # computation = first node -> completion
+           "latency_split_ms": {k: dict(zip(("p50", "p90", "p99"), (x * 1e3 for x in ctx.shard.percentiles(v))))
+                                for k, v in (("queueing", q_lat), ("computation", c_lat))},
+           "curve": curve, "roofline": roof,
+           "gpu_launches": int(st["kernel_launches"]), "tasks": int(st["tasks"]),
+           "rows_per_task": st["rows"] / max(1, st["tasks"]),
+           "sched_ns_per_task": st["sched_ns"] / max(1, st["tasks"]),
+           "clocks": clk.summary(), "persistent": bool(persistent), "policy": policy, "workers": workers}
+    if launch_log is not None and len(launch_log):
+        # launch duration vs rows (the tail of the timed region): where each class leaves its roof
+        hist = {}
+        for k in np.unique(launch_log["kclass"]):
+            m = launch_log["kclass"] == k
+            bs, sp = launch_log["b"][m], launch_log["span_ns"][m] / 1e3
+            edges = [1, 17, 33, 65, 129, 257, 385, 513]
+            rows = []
+            for lo_, hi_ in zip(edges[:-1], edges[1:]):
+                sel = (bs >= lo_) & (bs < hi_)
+                if sel.any():
+                    rows.append({"b": f"{lo_}-{hi_ - 1}", "launches": int(sel.sum()),
+                                 "mean_b": float(bs[sel].mean()), "span_us_mean": float(sp[sel].mean()),
+                                 "span_us_p10": float(np.percentile(sp[sel], 10)),
+                                 "span_us_p90": float(np.percentile(sp[sel], 90))})
+            hist[str(int(k))] = rows
+        out["span_vs_rows"] = hist
+    out["_engine"], out["_cells"], out["_w"], out["_trace"], out["_prep"] = e, cells, w, trace, prep
+    out["_persistent"], out["_policy"], out["_lookahead"], out["_workers"] = persistent, policy, lookahead, workers
+    return out
+
+
+def e2e_measure(ctx, a, wl, res, steps, warmup):
+    """The same metric through the public API with host buffers (submit from host, descriptors
+    H2D at every Schedule call inside bm_run, every request's final h D2H), host clock."""
+    bm, local = ctx.bm, ctx.local
+    n_req = res["requests_per_step"]
+    e2, cells2 = build_engine(bm, wl, res["_w"], local, max_requests=n_req + 64, lookahead=res["_lookahead"],
+                              time_kernels=0, keep=1, persistent=res["_persistent"], policy=res["_policy"],
+                              workers=res["_workers"], bucket_width=a.bucket_width)
     L, H = WL[wl]["layers"], WL[wl]["hidden"]
-    hbuf = torch.empty((n_req, L, H), dtype=torch.float32).pin_memory().numpy()
-    prep2 = e2.prepare_requests(trace, cells2)
-    for _ in range(max(1, a.warmup)):
+    hbuf = ctx.torch.empty((n_req, L, H), dtype=ctx.torch.float32).pin_memory().numpy()
+    prep2 = e2.prepare_requests(res["_trace"], cells2)
+    prep2.set_time_scale(1.0 / res["offered_rate_per_gpu"])
+    for _ in range(max(1, warmup)):
         fid = e2.submit_many(prep2)
         e2.run()
         e2.poll_array(n_req + 16)
         e2.read_results_many(fid, n_req, h=hbuf, release=True)
-    barrier()
+    ctx.barrier()
     t0 = time.perf_counter()
     rows0 = e2.stats()["rows"]
     ph = np.zeros(4)
-    for _ in range(a.steps):
+    for _ in range(steps):
         tp = [time.perf_counter()]
         fid = e2.submit_many(prep2)
         tp.append(time.perf_counter())
@@ -478,61 +644,191 @@ def main():
         e2.read_results_many(fid, n_req, h=hbuf, release=True)
         tp.append(time.perf_counter())
         ph += np.diff(tp)
-    e2e_s = allmax(time.perf_counter() - t0)
-    rows_e2e = (e2.stats()["rows"] - rows0) / a.steps
-    e2e = {"value": total / e2e_s, "unit": "requests/sec",
-           "h2d_bytes_per_step": int(rows_e2e * 16),
-           "d2h_bytes_per_step": int(n_req * L * H * 4),
-           "host_ms_per_step": dict(zip(("submit", "run", "poll", "read_results"),
-                                        (float(x) for x in ph * 1e3 / a.steps)))}
-    # ---- roofline of the dominant kernel (the LSTM / tree cell step), live CUDA events
-    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
-        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
-    hbm = peaks.get("hbm_gbs", 6650.0)
-    if st["timed_ms"] > 0:   # per-launch CUDA events (sampled launches) on the engine stream
-        t_kern = st["timed_ms"]
-        timing = ("CUDA events on the engine stream around a sample of cell-step launches (every 8th: "
-                  "events between launches would disable PDL overlap)")
-        kernel = {"lstm": "LSTM cell step: cell_pair_kernel (129-512 rows) + cell_step_sm100_kernel<EPI_LSTM>",
-                  "seq2seq": "Seq2Seq cell steps: 4 LSTM layers (cell_pair_kernel / cell_step_sm100_kernel<EPI_LSTM>) "
-                             "+ projection/argmax cell_step_sm100_kernel<EPI_PROJ>",
-                  "tree": "TreeLSTM cell steps: cell_step_sm100_kernel<EPI_LEAF> + <EPI_INTERNAL>"}[wl]
-    else:                    # persistent kernel: tasks run inside one launch
-        t_kern = st["span_ms"]
-        timing = ("persistent kernel: per-task device span (%globaltimer, first CTA ready .. last CTA "
-                  "done, summed over every task of the timed region); CUDA events bracket each whole step")
-        kernel = "lstm_persistent_kernel"
-    achieved = st["timed_bytes"] / (t_kern / 1e3) / 1e9 if t_kern > 0 else 0.0
-    tflops = st["timed_flops"] / (t_kern / 1e3) / 1e12 if t_kern > 0 else 0.0
-    bf16_peak = peaks.get("bf16_tflops", 1590.0)
-    traffic = load_traffic(wl) if not a.persistent else None
-    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
-            "traffic": traffic["dram_bytes_per_launch"] if traffic else None,
-            "traffic_unit": "bytes/launch (DRAM read+write, ncu, cold L2)",
-            "traffic_l2_to_sm": traffic["l2_to_sm_bytes_per_launch"] if traffic else None,
-            "traffic_source": traffic["file"] if traffic else None, "kernel": kernel, "timing": timing, "launches": st["timed_launches"],
-            "avg_launch_us": t_kern * 1e3 / max(1, st["timed_launches"]),
-            "avg_rows_per_task": st["rows"] / max(1, st["tasks"]), "tensor_tflops": tflops,
-            "tensor_frac": tflops / bf16_peak,
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)" if peaks else "fallback 6.65 TB/s",
-            # the same sampled launches timed on the device (%globaltimer: first CTA past its
-            # dependency wait .. last CTA done): excludes the serialisation the events impose
-            "device_span_us": (st["span_ms"] * 1e3 / st["span_launches"]) if st["span_launches"] else None,
-            "frac_device_span": ((st["timed_bytes"] / max(1, st["timed_launches"])) /
-                                 (st["span_ms"] / 1e3 / st["span_launches"]) / 1e9 / hbm)
-            if st["span_launches"] and st["timed_ms"] > 0 else None,
-            "note": ("algorithmic bytes count the 16.8 MB weight stream per step even when the persistent "
-                     "kernel keeps the weights on chip (so frac can exceed what DRAM moved)")}
+    e2e_s = ctx.allmax(time.perf_counter() - t0)
+    rows_e2e = (e2.stats()["rows"] - rows0) / steps
+    e2.close()
+    return {"value": n_req * steps * ctx.world / e2e_s, "unit": "requests/sec",
+            "h2d_bytes_per_step": int(rows_e2e * 16),
+            "d2h_bytes_per_step": int(n_req * L * H * 4),
+            "host_ms_per_step": dict(zip(("submit", "run", "poll", "read_results"),
+                                         (float(x) for x in ph * 1e3 / steps)))}
+
+
+def public(res):
+    return {k: v for k, v in res.items() if not k.startswith("_")}
+
+
+# ------------------------------------------------------------------------------ launcher
+def relaunch_under_torchrun(a):
+    """`--gpus N` (N > 1) without WORLD_SIZE: one process per GPU via torch.distributed.run."""
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    raise SystemExit(subprocess.call(cmd))
+
+
+# ------------------------------------------------------------------------------ main arm
+def main():
+    global LENGTHS, ENC_BMAX
+    a = parse()
+    ENC_BMAX = a.enc_bmax
+    LENGTHS = a.lengths if (a.workload == "lstm" and a.lengths != "identical") or \
+        (a.workload == "tree" and a.lengths == "identical") else "wmt"
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch_under_torchrun(a)
+    if world != a.gpus:
+        raise SystemExit(f"bench.py: --gpus {a.gpus} but WORLD_SIZE={world}: launch one process per GPU")
+    if a.impl == "reference":
+        return reference_arm(a)
+    import torch
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # one GPU per rank (NCCL over NVLink). With fewer GPUs than ranks (a functional check of the
+    # multi-rank path on one GPU) ranks share devices and the few collectives go over gloo.
+    ndev = max(1, torch.cuda.device_count())
+    local = local_rank % ndev
+    shared = world > ndev or a.dry
+    if not a.dry:
+        torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    from paper_conf_eurosys_gaoywl18_b200 import bm, shard
+    ctx = Ctx()
+    ctx.torch, ctx.bm, ctx.shard, ctx.dist = torch, bm, shard, dist
+    ctx.rank, ctx.world, ctx.local = rank, world, local
+    ctx.coll_dev = None if shared else torch.device("cuda", local)
+    ctx.peaks = load_peaks()
+    ctx.dry = a.dry
+
+    def barrier():
+        if not a.dry:
+            torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+    ctx.barrier = barrier
+    ctx.allmax = lambda x: shard.reduce_max(x, dist, device=ctx.coll_dev)
+    ctx.allmin = lambda x: -shard.reduce_max(-x, dist, device=ctx.coll_dev)
+
+    wl = a.workload
+    n_req = a.reqs or WL[wl]["reqs"]
+    res = run_workload(ctx, a, wl, n_req, a.steps, a.warmup, headline=True)
+    e2e = None if a.dry else e2e_measure(ctx, a, wl, res, a.steps, a.warmup)
+    e, cells = res["_engine"], res["_cells"]
     bound = None
     if wl == "lstm" and LENGTHS == "fixed24":
-        # L679-L681: with every request 24 steps long the throughput bound is
-        # bmax / (24 x t_step(bmax)); t_step measured here on full 512-row tasks, back to back
-        rng = np.random.default_rng(5)
-        b = 512
-        slots = rng.choice(1 << 16, size=b, replace=False).astype(np.int32)
-        rows = np.stack([rng.integers(3, WL[wl]["vocab"], size=b), np.zeros(b), slots,
-                         (np.arange(b) % 2) * bm.ROW_PARITY], 1)
-        cid = cells[gen.CHAIN][0]
+        bound = fixed24_bound(ctx, e, cells, res["value"])
+    if wl == "tree" and LENGTHS == "identical":
+        bound = identical_tree_bound(ctx, e, cells, res["value"])
+    e.close()
+    extras = {}
+    extra = a.extra
+    if extra == "auto":
+        extra = "seq2seq,tree" if (wl == "lstm" and world == 1 and LENGTHS == "wmt" and a.policy == "cellular"
+                                   and a.workers == 1 and a.persistent <= 0 and not a.quick
+                                   and not a.dry) else "none"
+    for x in [s for s in extra.split(",") if s and s != "none" and s != wl]:
+        r = run_workload(ctx, a, x, EXTRA_REQS[x], EXTRA_STEPS, 1, headline=False)
+        r["_engine"].close()
+        r = public(r)
+        r["config"] = WL[x]["config"]
+        r["steps"], r["warmup"] = EXTRA_STEPS, 1
+        extras[x] = r
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline and not a.dry:
+        cpu = cpu_oracle(wl, a.cpu_seconds)
+    if rank == 0:
+        r = public(res)
+        line = {"metric": METRIC, "value": r["value"], "unit": "requests/sec", "n_gpus": world, "steps": a.steps,
+                "warmup": a.warmup, "ms_per_step": r["ms_per_step"], "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+                "config": {"workload": WL[wl]["config"] if LENGTHS == "wmt" else
+                           (WL[wl]["config"].replace("WMT-like lengths", f"Fig. 11 lengths '{LENGTHS}'")
+                            if wl == "lstm" else WL[wl]["config"] + "; identical complete 16-leaf trees (Fig. 15)"),
+                           "requests_per_step": n_req, "offered_rate_per_gpu": r["offered_rate_per_gpu"],
+                           "p90_bound_ms": r["p90_bound_ms"], "p90_bound_kind": r["p90_bound_kind"],
+                           "max_offered_rate_under": r["max_offered_rate_under"],
+                           "saturation_burst_rate_per_gpu": r["saturation_burst_rate_per_gpu"],
+                           "lookahead_k": r["lookahead_k"],
+                           "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
+                                 "step (serving)", "parallelism": f"request-sharded x{world}",
+                           "persistent_kernel": r["persistent"], "workers_per_gpu": r["workers"],
+                           "bmax": ({"encoder": ENC_BMAX, "decoder": 256} if wl == "seq2seq" else
+                                    (512 if wl == "lstm" else 64)),
+                           "policy": ("cellular batching (Algorithm 1)" if r["policy"] == bm.POLICY_CELLULAR else
+                                      f"graph-batching baseline: padding + bucketing, width {a.bucket_width}, "
+                                      "round robin over buckets (L427)")},
+                "latency_ms": r["latency_ms"], "latency_split_ms": r["latency_split_ms"],
+                "achieved_over_offered": r["achieved_over_offered"],
+                "curve": r["curve"], "e2e": e2e, "roofline": r["roofline"], "cpu_baseline": cpu,
+                "analytic_bound": bound, "clocks": r["clocks"], "gpu_launches": r["gpu_launches"],
+                "tasks": r["tasks"], "rows_per_task": r["rows_per_task"],
+                "sched_ns_per_task": r["sched_ns_per_task"], "span_vs_rows": r.get("span_vs_rows"),
+                "extra_workloads": extras or None,
+                "comm": {"backend": dist.get_backend() if dist is not None else None, "world_size": world,
+                         "weights": "broadcast once from rank 0, adopted in place by bm_load_cell" if world > 1
+                         else "loaded from host", "per_step_collectives": 0}}
+        if a.dry:
+            line["dry"] = "BM_CLOCK_DRY functional check: value and latencies are in virtual ticks, no kernels ran"
+            line["dtype"] = None
+        s = json.dumps(line)
+        print(s, flush=True)
+        if a.out:
+            with open(a.out, "w") as f:
+                f.write(s + "\n")
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+def fixed24_bound(ctx, e, cells, value):
+    """L679-L681: with every request 24 steps long the throughput bound is bmax / (24 x
+    t_step(bmax)); t_step measured here on full 512-row tasks, back to back."""
+    bm, torch = ctx.bm, ctx.torch
+    stream = torch.cuda.ExternalStream(e.stream())
+    rng = np.random.default_rng(5)
+    b = 512
+    slots = rng.choice(1 << 16, size=b, replace=False).astype(np.int32)
+    rows = np.stack([rng.integers(3, WL["lstm"]["vocab"], size=b), np.zeros(b), slots,
+                     (np.arange(b) % 2) * bm.ROW_PARITY], 1)
+    cid = cells[gen.CHAIN][0]
+    for _ in range(5):
+        e.cell_step(cid, rows, sync=False)
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for _ in range(50):
+        e.cell_step(cid, rows, sync=False)
+    ev1.record(stream)
+    ev1.synchronize()
+    t_step = ev0.elapsed_time(ev1) / 50 / 1e3
+    b_req = b / (24 * t_step) * ctx.world
+    return {"t_step_b512_us": t_step * 1e6, "bound_req_s": b_req, "fraction_of_bound": value / b_req,
+            "paper": "BatchMaker at ~87% of 27,136 req/s on V100 (L679-L681)"}
+
+
+def identical_tree_bound(ctx, e, cells, value):
+    """Fig. 15 (L857): identical complete 16-leaf trees against a hard-coded ideal that packs
+    every level of 64/16 = 4 trees into full tasks: per tree 16 leaf rows + 15 internal rows,
+    i.e. 16/64 of a 64-row leaf task + 15/64 of a 64-row internal task."""
+    torch = ctx.torch
+    stream = torch.cuda.ExternalStream(e.stream())
+    rng = np.random.default_rng(5)
+    b = 64
+    slots = rng.choice(1 << 16, size=3 * b, replace=False).astype(np.int32)
+    leaf_rows = np.stack([rng.integers(3, WL["tree"]["vocab"], size=b), np.zeros(b), slots[:b], np.zeros(b)], 1)
+    int_rows = np.stack([slots[b:2 * b], slots[2 * b:], slots[:b], np.zeros(b)], 1)
+    lf, it = cells[gen.TREE]
+    t = {}
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for name, cid, rows in (("leaf", lf, leaf_rows), ("internal", it, int_rows)):
         for _ in range(5):
             e.cell_step(cid, rows, sync=False)
         torch.cuda.synchronize()
@@ -541,75 +837,11 @@ def main():
             e.cell_step(cid, rows, sync=False)
         ev1.record(stream)
         ev1.synchronize()
-        t_step = ev0.elapsed_time(ev1) / 50 / 1e3
-        b_req = b / (24 * t_step) * world
-        bound = {"t_step_b512_us": t_step * 1e6, "bound_req_s": b_req, "fraction_of_bound": value / b_req,
-                 "paper": "BatchMaker at ~87% of 27,136 req/s on V100 (L679-L681)"}
-    if wl == "tree" and LENGTHS == "identical":
-        # Fig. 15 (L857): identical complete 16-leaf trees against a hard-coded ideal that packs
-        # every level of 64/16 = 4 trees into full tasks: per tree 16 leaf rows + 15 internal
-        # rows, i.e. 16/64 of a 64-row leaf task + 15/64 of a 64-row internal task
-        rng = np.random.default_rng(5)
-        b = 64
-        slots = rng.choice(1 << 16, size=3 * b, replace=False).astype(np.int32)
-        leaf_rows = np.stack([rng.integers(3, WL[wl]["vocab"], size=b), np.zeros(b), slots[:b], np.zeros(b)], 1)
-        int_rows = np.stack([slots[b:2 * b], slots[2 * b:], slots[:b], np.zeros(b)], 1)
-        lf, it = cells[gen.TREE]
-        t = {}
-        for name, cid, rows in (("leaf", lf, leaf_rows), ("internal", it, int_rows)):
-            for _ in range(5):
-                e.cell_step(cid, rows, sync=False)
-            torch.cuda.synchronize()
-            ev0.record(stream)
-            for _ in range(50):
-                e.cell_step(cid, rows, sync=False)
-            ev1.record(stream)
-            ev1.synchronize()
-            t[name] = ev0.elapsed_time(ev1) / 50 / 1e3
-        ideal = world / (16 / b * t["leaf"] + 15 / b * t["internal"])
-        bound = {"t_leaf_b64_us": t["leaf"] * 1e6, "t_internal_b64_us": t["internal"] * 1e6,
-                 "ideal_req_s": ideal, "fraction_of_ideal": value / ideal,
-                 "paper": "BatchMaker peak ~30% below the hard-coded ideal (L857)"}
-    cpu = None
-    if rank == 0 and world == 1 and not a.no_cpu_baseline:
-        cpu = cpu_oracle(wl, a.cpu_seconds)
-    if rank == 0:
-        line = {"metric": METRIC, "value": value, "unit": "requests/sec", "n_gpus": world, "steps": a.steps,
-                "warmup": a.warmup, "ms_per_step": t_max * 1e3 / a.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-                "config": {"workload": WL[wl]["config"] if LENGTHS == "wmt" else
-                           (WL[wl]["config"].replace("WMT-like lengths", f"Fig. 11 lengths '{LENGTHS}'")
-                            if wl == "lstm" else WL[wl]["config"] + "; identical complete 16-leaf trees (Fig. 15)"),
-                           "requests_per_step": n_req,
-                           "offered_rate_per_gpu": lam_star, "p90_bound_ms": bound_ms,
-                           "p90_bound_kind": bound_kind,
-                           "max_offered_rate_under": bounds if a.rate <= 0 else None,
-                           "saturation_burst_rate_per_gpu": mu, "lookahead_k": a.lookahead,
-                           "l2": "256 MB buffer written between timed steps; weights L2-resident within a "
-                                 "step (serving)", "parallelism": f"request-sharded x{world}",
-                           "persistent_kernel": bool(a.persistent), "workers_per_gpu": a.workers,
-                           "bmax": ({"encoder": ENC_BMAX, "decoder": 256} if wl == "seq2seq" else
-                                    (512 if wl == "lstm" else 64)),
-                           "policy": ("cellular batching (Algorithm 1)" if policy == bm.POLICY_CELLULAR else
-                                      f"graph-batching baseline: padding + bucketing, width {a.bucket_width}, "
-                                      "round robin over buckets (L427)")},
-                "latency_ms": {"p50": p50 * 1e3, "p90": p90 * 1e3, "p99": p99 * 1e3},
-                # Fig. 9's decomposition (L597): queueing = arrival -> first node scheduled,
-                # computation = first node -> completion
-                "latency_split_ms": {k: dict(zip(("p50", "p90", "p99"), (x * 1e3 for x in shard.percentiles(v))))
-                                     for k, v in (("queueing", q_lat), ("computation", c_lat))},
-                "curve": curve, "e2e": e2e, "roofline": roof, "cpu_baseline": cpu, "analytic_bound": bound,
-                "clocks": clk.summary(), "gpu_launches": int(st["kernel_launches"]),
-                "sched_ns_per_task": st["sched_ns"] / max(1, st["tasks"])}
-        s = json.dumps(line)
-        print(s, flush=True)
-        if a.out:
-            with open(a.out, "w") as f:
-                f.write(s + "\n")
-    e.close()
-    e2.close()
-    if dist is not None:
-        dist.destroy_process_group()
+        t[name] = ev0.elapsed_time(ev1) / 50 / 1e3
+    ideal = ctx.world / (16 / b * t["leaf"] + 15 / b * t["internal"])
+    return {"t_leaf_b64_us": t["leaf"] * 1e6, "t_internal_b64_us": t["internal"] * 1e6,
+            "ideal_req_s": ideal, "fraction_of_ideal": value / ideal,
+            "paper": "BatchMaker peak ~30% below the hard-coded ideal (L857)"}
 
 
 if __name__ == "__main__":

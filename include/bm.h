@@ -14,9 +14,11 @@
  *   Schedule(worker) runs when a worker becomes idle ............................. L371 (§4.3)
  *   completion is detected by polling a signal counter in pinned host memory .... L393-L395 (§5)
  *
- * Threading: an engine is single-threaded by contract (all calls from one thread), except
- * that bm_poll may be called from one dedicated polling thread concurrently with the
- * others. Different engines (one per GPU) are independent.
+ * Threading: every call on an engine takes that engine's lock, so calls from several threads
+ * are serialised and safe. In particular bm_poll may run on a dedicated polling thread (the
+ * paper's poll thread, L395) while another thread submits and schedules; bm_run takes the
+ * lock once per round of its event loop, so a concurrent bm_poll interleaves between rounds.
+ * Different engines (one per GPU) are independent.
  *
  * Error behaviour: every call returns a bm_status. BM_E_CUDA is sticky: after it every
  * call that touches the device returns BM_E_CUDA again and the engine can only be
@@ -76,7 +78,8 @@ typedef struct {
   int max_decode_len;        /* decoder tokens kept per request (result buffer)           */
   int keep_results;          /* 1: results stay readable until bm_release; 0: auto-free  */
   int record_logits;         /* debug: keep every decode step's logits (parity tests)     */
-  int time_kernels;          /* 1: CUDA-event time every cell-step launch (bench roofline)*/
+  int time_kernels;          /* 1: device-time EVERY kernel launch (per-kernel roofline,  */
+                             /* bm_stats.k_*, bm_read_launch_log)                          */
   int record_log;            /* 1: keep the task log for bm_read_log (default 1)          */
   int persistent;            /* 1: bm_run serves an engine whose only cell is a 1-layer   */
                              /* LSTM with one persistent, weight-stationary kernel (its   */
@@ -95,6 +98,8 @@ typedef struct {
                              /* request sharding's one worker per GPU (default). >1 needs */
                              /* policy CELLULAR and persistent 0; the bf16 LSTM launches  */
                              /* then use a <= 113 KB plan so two workers' CTAs share SMs. */
+  double roof_hbm_gbs;       /* time_kernels: the roofline denominators (bench.py passes     */
+  double roof_tc_tflops;     /* MEASURED_PEAKS.json); 0 = bm_stats.k_roof_* stay 0          */
 } bm_config;
 
 enum {
@@ -125,9 +130,13 @@ typedef struct {
   int priority;   /* larger = scheduled first among equals (L339, Alg. 1 line 10)       */
 } bm_cell_desc;
 
-/* Weights in the paper/oracle layout, row-major fp32, host pointers (copied; the caller
- * keeps ownership and may free them after the call). In BF16 precision they are rounded
- * to bf16 (round-to-nearest-even) and packed on the device by the library.
+/* Weights in the paper/oracle layout, row-major fp32 (startup loads each cell and "embeds"
+ * its weights, L319). Each pointer may be a HOST pointer (copied up) or a DEVICE pointer on
+ * the engine's device (adopted in place: the packing kernels read it directly, so weights
+ * broadcast once with NCCL land without a host round trip); a device pointer
+ * of another device is BM_E_INVAL. The library keeps its own packed copy; the caller keeps
+ * ownership and may free the arrays after the call. In BF16 precision they are rounded to
+ * bf16 (round-to-nearest-even) and packed on the device by the library.
  *   BM_CELL_LSTM / _PROJ: W[l] = [4h, 2h] acting on the column [x; h], gate row blocks
  *                         (i, f, g, o); b[l] = [4h]; E = [vocab, h];
  *                         _PROJ adds W_out = [vocab, h], b_out = [vocab].
@@ -175,8 +184,12 @@ typedef struct {
 } bm_request;
 
 /* Admit a request (unfold, A1). All arrays are copied. The request becomes visible to the
- * scheduler once the clock reaches `arrival`. *req_id = admission index (0, 1, 2, ...).
- * Errors: BM_E_INVAL (bad cell kinds, token out of range, tree not binary/post-order),
+ * scheduler once the clock reaches `arrival` ("When a new request arrives, the request
+ * processor runs the user-code to unfold the recursion", L323). *req_id = admission index
+ * (0, 1, 2, ...). Requests not yet admitted form an arrival stream: `arrival` must be >= the
+ * arrival of every earlier-submitted request that is still pending (BM_E_INVAL otherwise).
+ * Errors: BM_E_INVAL (bad cell kinds, token out of range, tree not binary/post-order,
+ * arrival earlier than a pending request's),
  * BM_E_FULL (request table full; retry after retiring), BM_E_STATE. */
 bm_status bm_submit(bm_engine* e, const bm_request* r, uint64_t* req_id);
 
@@ -223,11 +236,11 @@ bm_status bm_read_result(bm_engine* e, uint64_t req_id, bm_result* dst);
 bm_status bm_release(bm_engine* e, uint64_t req_id);
 
 /* Bulk result read for the consecutive ids [first_id, first_id + n), all completed and kept:
- * one device->host copy per contiguous table range. h: [n][pool_layers][hidden] fp32 or
+ * one device->host copy per contiguous table range. h, c: [n][pool_layers][hidden] fp32 or
  * NULL; tokens: [n][max_decode_len] or NULL (entries past a request's last emitted token are
  * -1). Then releases them if release != 0. */
-bm_status bm_read_results_many(bm_engine* e, uint64_t first_id, int n, float* h, int32_t* tokens,
-                               int release);
+bm_status bm_read_results_many(bm_engine* e, uint64_t first_id, int n, float* h, float* c,
+                               int32_t* tokens, int release);
 
 /* Task log (replay parity, P9): one record per launched task, rows flattened. */
 typedef struct {
@@ -280,26 +293,58 @@ bm_status bm_result_rows(bm_engine* e, const int32_t* res_idx, int n, float* h, 
 /* Device feed tokens tok[slot] (decoder) in/out. */
 bm_status bm_tokens(bm_engine* e, const int32_t* slots, int n, int32_t* inout, int write);
 
-/* ---------------------------------------------------------------- measurement */
+/* ---------------------------------------------------------------- measurement
+ * Per-kernel roofline accounting (time_kernels = 1). EVERY launch is timed on the device: its
+ * span runs from the first CTA past its dependency wait (the point where the launch's
+ * dependent work may begin; under PDL its setup overlaps the previous launch) to the last CTA
+ * done (%globaltimer), accumulated per kernel class by the launch's last CTA. The host adds
+ * the same launch's ALGORITHMIC bytes and flops (weights streamed once,
+ * gathered operand rows, state read/written; padding not counted) to the same class, so
+ * bytes, flops and time always cover one population. k_roof_* sum, per launch, the time the
+ * launch would take at the roof: bytes / roof_hbm_gbs, flops / roof_tc_tflops, and the larger
+ * of the two (the launch's binding roof: HBM below the ridge, tensor above). */
+enum {
+  BM_K_LSTM_PAIR = 0,   /* cell_pair_kernel: LSTM layer, tcgen05 cta_group::2 (129-512 rows) */
+  BM_K_LSTM = 1,        /* cell_step_sm100_kernel<EPI_LSTM>                                  */
+  BM_K_LEAF = 2,        /* cell_step_sm100_kernel<EPI_LEAF>                                  */
+  BM_K_INTERNAL = 3,    /* cell_step_sm100_kernel<EPI_INTERNAL>                              */
+  BM_K_PROJ = 4,        /* decoder projection + argmax                                       */
+  BM_K_SIMT = 5,        /* fp32 SIMT parity path (all cell kinds)                            */
+  BM_K_PERSISTENT = 6,  /* persistent weight-stationary LSTM: one "launch" = one task        */
+  BM_K_CLASSES = 8
+};
+
 typedef struct {
   uint64_t tasks;            /* tasks launched                                           */
   uint64_t rows;             /* rows (cell nodes) executed                               */
   uint64_t kernel_launches;  /* our kernels launched                                     */
-  uint64_t timed_launches;   /* launches with CUDA-event timing (time_kernels)           */
-  double timed_ms;           /* sum of those launches' device durations                  */
-  double timed_bytes;        /* sum of their algorithmic bytes     */
-  double timed_flops;        /* sum of their algorithmic flops                           */
   double sched_ns;           /* host time spent in Schedule/Batch                        */
   uint64_t schedule_calls;
-  double span_ms;            /* same launches, device-side span (first CTA start .. last  */
-                             /* CTA end, %globaltimer): excludes host launch latency      */
   double launch_ns;          /* host time spent staging descriptors and issuing launches  */
   double retire_ns;          /* host time spent retiring finished tasks (Retire, A4)      */
-  uint64_t span_launches;    /* launches whose device span is in span_ms                  */
+  uint64_t k_launches[BM_K_CLASSES];      /* launches issued, per class                  */
+  uint64_t k_span_launches[BM_K_CLASSES]; /* launches whose device span landed (equal to */
+                                          /* k_launches once the device is idle)          */
+  double k_span_ms[BM_K_CLASSES];         /* sum of device spans                         */
+  double k_rows[BM_K_CLASSES];            /* sum of rows (b) over the launches           */
+  double k_bytes[BM_K_CLASSES];           /* sum of algorithmic bytes                    */
+  double k_flops[BM_K_CLASSES];           /* sum of algorithmic flops                    */
+  double k_roof_hbm_ms[BM_K_CLASSES];     /* sum of bytes / roof_hbm_gbs                 */
+  double k_roof_tc_ms[BM_K_CLASSES];      /* sum of flops / roof_tc_tflops               */
+  double k_roof_ms[BM_K_CLASSES];         /* sum of max(the two) per launch              */
 } bm_stats;
 
 bm_status bm_get_stats(bm_engine* e, bm_stats* out);
 bm_status bm_reset_stats(bm_engine* e);
+
+/* Launch log (time_kernels = 1): the last <= 65536 launches since bm_reset_stats, oldest
+ * first: kernel class, rows, device span in ns (0 if not landed). Synchronises the stream. */
+typedef struct {
+  int kclass;
+  int b;
+  uint64_t span_ns;
+} bm_launch_record;
+bm_status bm_read_launch_log(bm_engine* e, bm_launch_record* out, int cap, int* n);
 
 /* Device stream the engine launches on (cudaStream_t as void*), so callers can bracket
  * runs with CUDA events on that stream. */

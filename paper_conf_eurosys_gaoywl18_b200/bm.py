@@ -36,7 +36,8 @@ class Config(C.Structure):
         "device", "precision", "clock", "hidden", "pool_layers", "max_slots", "max_requests",
         "max_tasks_to_submit", "min_followon_batch", "schedule_when_outstanding_leq",
         "max_decode_len", "keep_results", "record_logits", "time_kernels", "record_log",
-        "persistent", "policy", "bucket_width", "workers")]
+        "persistent", "policy", "bucket_width", "workers")] + [
+        ("roof_hbm_gbs", C.c_double), ("roof_tc_tflops", C.c_double)]
 
 
 class CellDesc(C.Structure):
@@ -80,13 +81,24 @@ class StepRow(C.Structure):
     _fields_ = [("a", C.c_int32), ("b", C.c_int32), ("slot", C.c_int32), ("flags", C.c_int32)]
 
 
+K_LSTM_PAIR, K_LSTM, K_LEAF, K_INTERNAL, K_PROJ, K_SIMT, K_PERSISTENT, K_CLASSES = 0, 1, 2, 3, 4, 5, 6, 8
+K_NAMES = {K_LSTM_PAIR: "cell_pair_kernel (LSTM, cta_group::2)", K_LSTM: "cell_step_sm100_kernel<EPI_LSTM>",
+           K_LEAF: "cell_step_sm100_kernel<EPI_LEAF>", K_INTERNAL: "cell_step_sm100_kernel<EPI_INTERNAL>",
+           K_PROJ: "cell_step_sm100_kernel<EPI_PROJ> (projection + argmax)", K_SIMT: "fp32 SIMT cell kernels",
+           K_PERSISTENT: "lstm_persistent_kernel (per task)"}
+
+
 class Stats(C.Structure):
     _fields_ = [("tasks", C.c_uint64), ("rows", C.c_uint64), ("kernel_launches", C.c_uint64),
-                ("timed_launches", C.c_uint64), ("timed_ms", C.c_double),
-                ("timed_bytes", C.c_double), ("timed_flops", C.c_double),
-                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64), ("span_ms", C.c_double),
+                ("sched_ns", C.c_double), ("schedule_calls", C.c_uint64),
                 ("launch_ns", C.c_double), ("retire_ns", C.c_double),
-                ("span_launches", C.c_uint64)]
+                ("k_launches", C.c_uint64 * K_CLASSES), ("k_span_launches", C.c_uint64 * K_CLASSES)] + [
+        (n, C.c_double * K_CLASSES) for n in ("k_span_ms", "k_rows", "k_bytes", "k_flops", "k_roof_hbm_ms",
+                                              "k_roof_tc_ms", "k_roof_ms")]
+
+
+class LaunchRecord(C.Structure):
+    _fields_ = [("kclass", C.c_int), ("b", C.c_int), ("span_ns", C.c_uint64)]
 
 
 # exported symbols (tests/test_abi.py checks them against include/bm.h)
@@ -107,7 +119,7 @@ _SIGS = {
     "bm_read_result": (C.c_int, [_P, C.c_uint64, C.POINTER(Result)]),
     "bm_release": (C.c_int, [_P, C.c_uint64]),
     "bm_read_results_many": (C.c_int, [_P, C.c_uint64, C.c_int, C.POINTER(C.c_float),
-                                       C.POINTER(C.c_int32), C.c_int]),
+                                       C.POINTER(C.c_float), C.POINTER(C.c_int32), C.c_int]),
     "bm_read_log": (C.c_int, [_P, C.POINTER(TaskRecord), C.c_int, C.POINTER(C.c_int)]),
     "bm_read_log_rows": (C.c_int, [_P, C.POINTER(RowRecord), C.c_int, C.POINTER(C.c_int)]),
     "bm_cell_step": (C.c_int, [_P, C.c_int, C.POINTER(StepRow), C.c_int, C.c_int]),
@@ -120,6 +132,7 @@ _SIGS = {
     "bm_tokens": (C.c_int, [_P, C.POINTER(C.c_int32), C.c_int, C.POINTER(C.c_int32), C.c_int]),
     "bm_get_stats": (C.c_int, [_P, C.POINTER(Stats)]),
     "bm_reset_stats": (C.c_int, [_P]),
+    "bm_read_launch_log": (C.c_int, [_P, C.POINTER(LaunchRecord), C.c_int, C.POINTER(C.c_int)]),
     "bm_stream": (C.c_void_p, [_P]),
 }
 for _name, (_res, _args) in _SIGS.items():
@@ -131,6 +144,14 @@ for _name, (_res, _args) in _SIGS.items():
 class _Prepared:
     def __init__(self, arr, toks, lr):
         self.arr, self.toks, self.lr = arr, toks, lr
+        # numpy view of the arrival field of every bm_request (no per-request Python objects)
+        self.arrival = np.ndarray((len(arr),), np.float64, buffer=arr, offset=Request.arrival.offset,
+                                  strides=(C.sizeof(Request),))
+        self.base_arrival = self.arrival.copy()
+
+    def set_time_scale(self, scale: float):
+        """arrival_i = base arrival_i * scale (a unit-rate Poisson trace becomes rate 1/scale)."""
+        self.arrival[:] = self.base_arrival * scale
 
 
 class BMError(RuntimeError):
@@ -165,7 +186,7 @@ def default_config(**kw) -> Config:
     cfg = Config()
     lib.bm_config_default(C.byref(cfg))
     for k, v in kw.items():
-        setattr(cfg, k, int(v))
+        setattr(cfg, k, float(v) if k.startswith("roof_") else int(v))
     return cfg
 
 
@@ -200,15 +221,23 @@ class Engine:
     def load_cell(self, kind: int, layers: int, vocab: int, max_batch: int, priority: int,
                   W: Sequence[np.ndarray], b: Sequence[np.ndarray], E: Optional[np.ndarray] = None,
                   W_out: Optional[np.ndarray] = None, b_out: Optional[np.ndarray] = None) -> int:
+        """Arrays are numpy (host, copied up) or fp32 CUDA tensors on the engine's device
+        (anything with data_ptr(): adopted in place, e.g. after an NCCL broadcast)."""
         d = CellDesc(kind, self.cfg.hidden, layers, vocab, max_batch, priority)
-        Ws = [_f32(x) for x in W]
-        bs = [_f32(x) for x in b]
-        Wa = (C.POINTER(C.c_float) * len(Ws))(*[_fp(x) for x in Ws])
-        ba = (C.POINTER(C.c_float) * len(bs))(*[_fp(x) for x in bs])
-        Ea = _f32(E) if E is not None else None
-        Wo = _f32(W_out) if W_out is not None else None
-        bo = _f32(b_out) if b_out is not None else None
-        w = Weights(Wa, ba, _fp(Ea), _fp(Wo), _fp(bo))
+        keep = []
+
+        def ptr(x):
+            if x is None:
+                return None
+            if hasattr(x, "data_ptr"):
+                keep.append(x)
+                return C.cast(C.c_void_p(x.data_ptr()), C.POINTER(C.c_float))
+            a = _f32(x)
+            keep.append(a)
+            return _fp(a)
+        Wa = (C.POINTER(C.c_float) * len(W))(*[ptr(x) for x in W])
+        ba = (C.POINTER(C.c_float) * len(b))(*[ptr(x) for x in b])
+        w = Weights(Wa, ba, ptr(E), ptr(W_out), ptr(b_out))
         cid = C.c_int()
         _ck(lib.bm_load_cell(self.h, C.byref(d), C.byref(w), C.byref(cid)), "bm_load_cell")
         return cid.value
@@ -265,8 +294,9 @@ class Engine:
         return first.value
 
     def read_results_many(self, first_id: int, n: int, h: Optional[np.ndarray] = None,
-                          tokens: Optional[np.ndarray] = None, release: bool = True):
-        _ck(lib.bm_read_results_many(self.h, first_id, n, _fp(h), _ip(tokens), 1 if release else 0),
+                          tokens: Optional[np.ndarray] = None, release: bool = True,
+                          c: Optional[np.ndarray] = None):
+        _ck(lib.bm_read_results_many(self.h, first_id, n, _fp(h), _fp(c), _ip(tokens), 1 if release else 0),
             "bm_read_results_many")
 
     def schedule_step(self) -> int:
@@ -372,10 +402,24 @@ class Engine:
     def stats(self) -> dict:
         st = Stats()
         _ck(lib.bm_get_stats(self.h, C.byref(st)), "bm_get_stats")
-        return {k: getattr(st, k) for k, _ in Stats._fields_}
+        out = {}
+        for k, _ in Stats._fields_:
+            v = getattr(st, k)
+            out[k] = list(v) if k.startswith("k_") else v
+        return out
 
     def reset_stats(self):
         _ck(lib.bm_reset_stats(self.h), "bm_reset_stats")
+
+    _LAUNCH_DT = np.dtype([("kclass", "<i4"), ("b", "<i4"), ("span_ns", "<u8")])
+
+    def launch_log(self, cap: int = 1 << 16) -> np.ndarray:
+        """bm_read_launch_log: (kernel class, rows, device span ns) of the last launches."""
+        out = np.zeros(cap, dtype=self._LAUNCH_DT)
+        n = C.c_int()
+        _ck(lib.bm_read_launch_log(self.h, out.ctypes.data_as(C.POINTER(LaunchRecord)), cap, C.byref(n)),
+            "bm_read_launch_log")
+        return out[:n.value]
 
     def stream(self) -> int:
         return int(lib.bm_stream(self.h) or 0)

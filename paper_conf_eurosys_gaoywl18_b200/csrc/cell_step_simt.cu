@@ -46,8 +46,35 @@ __device__ __forceinline__ const float* seg_src(const StepArgs& p, const RowDesc
 
 // Gate GEMM + fused epilogue. CTA tile: 32 units (all G gates of each) x 32 batch columns.
 // Thread t: unit j = t % 32, columns 4 * (t / 32) .. +3.
+// Device span of a launch (time_kernels, include/bm.h BM_K_SIMT): first CTA start .. last CTA
+// done (%globaltimer), accumulated by the last CTA.
+__device__ __forceinline__ unsigned long long simt_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void span_begin(const StepArgs& p) {
+  if (p.span != nullptr && threadIdx.x == 0) atomicMin(p.span, simt_now());
+}
+__device__ __forceinline__ void span_end(const StepArgs& p) {
+  if (p.span == nullptr) return;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long total = gridDim.x * gridDim.y * gridDim.z;
+    if (atomicAdd(p.span + 1, 1ull) == total - 1) {
+      const unsigned long long t0 = atomicExch(p.span, ~0ull);
+      atomicExch(p.span + 1, 0ull);
+      const unsigned long long dt = simt_now() - t0;
+      atomicAdd(p.span_acc, dt);
+      atomicAdd(p.span_acc + 1, 1ull);
+      if (p.span_log != nullptr) *p.span_log = dt;
+    }
+  }
+}
+
 template <int EPI>
-__global__ void __launch_bounds__(kThreads) cell_step_simt_kernel(const __grid_constant__ StepArgs p) {
+__device__ __forceinline__ void cell_step_simt_body(const StepArgs& p) {
   constexpr int G = EPI == EPI_LSTM ? 4 : EPI == EPI_LEAF ? 3 : 5;
   __shared__ float Ws[G * kTU][kTK + 1];
   __shared__ float Xs[kTC][kTK + 1];
@@ -150,7 +177,14 @@ __global__ void __launch_bounds__(kThreads) cell_step_simt_kernel(const __grid_c
 // Projection + argmax, fp32. CTA: 128 vocab rows x 32 columns; per-column argmax packed into a
 // 64-bit key (ordered value, inverted index) and reduced across CTAs with atomicMax; the last CTA
 // publishes the tokens (same protocol as the tcgen05 kernel).
-__global__ void __launch_bounds__(kThreads) proj_simt_kernel(const __grid_constant__ StepArgs p) {
+template <int EPI>
+__global__ void __launch_bounds__(kThreads) cell_step_simt_kernel(const __grid_constant__ StepArgs p) {
+  span_begin(p);
+  cell_step_simt_body<EPI>(p);
+  span_end(p);
+}
+
+__device__ __forceinline__ void proj_simt_body(const StepArgs& p) {
   __shared__ float Ws[128][kTK + 1];
   __shared__ float Xs[kTC][kTK + 1];
   __shared__ const float* src[kTC];
@@ -257,6 +291,12 @@ __global__ void __launch_bounds__(kThreads) proj_simt_kernel(const __grid_consta
     }
     if (tid == 0) *p.done_ctas = 0;
   }
+}
+
+__global__ void __launch_bounds__(kThreads) proj_simt_kernel(const __grid_constant__ StepArgs p) {
+  span_begin(p);
+  proj_simt_body(p);
+  span_end(p);
 }
 
 // fp32 paper layout [G*H][K] (row g*H + u) -> packed [H*G][K] (row u*G + g), bf16 or fp32.

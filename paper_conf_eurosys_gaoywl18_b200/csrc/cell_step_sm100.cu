@@ -753,8 +753,10 @@ __global__ void __launch_bounds__(kThreads, 2)
       if (atomicAdd(p.span + 1, 1ull) == total - 1) {
         const unsigned long long t0 = atomicExch(p.span, ~0ull);
         atomicExch(p.span + 1, 0ull);
-        atomicAdd(p.span_acc, gtimer() - t0);
+        const unsigned long long dt = gtimer() - t0;
+        atomicAdd(p.span_acc, dt);
         atomicAdd(p.span_acc + 1, 1ull);
+        if (p.span_log != nullptr) *p.span_log = dt;
       }
     }
   }
@@ -1310,8 +1312,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (atomicAdd(p.span + 1, 1ull) == total - 1) {
         const unsigned long long t0 = atomicExch(p.span, ~0ull);
         atomicExch(p.span + 1, 0ull);
-        atomicAdd(p.span_acc, gtimer() - t0);
+        const unsigned long long dt = gtimer() - t0;
+        atomicAdd(p.span_acc, dt);
         atomicAdd(p.span_acc + 1, 1ull);
+        if (p.span_log != nullptr) *p.span_log = dt;
       }
     }
   }
@@ -1439,21 +1443,28 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
 
 }  // namespace
 
-cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st) {
-  if (a.b <= 0) return cudaSuccess;
+cudaError_t launch_cell_step_sm100(const StepArgs& a0, const RowDesc* rows_host, cudaStream_t st, int* kclass) {
+  if (a0.b <= 0) return cudaSuccess;
+  StepArgs a = a0;
+  // kernel classes (include/bm.h BM_K_*): 0 pair LSTM, 1 LSTM, 2 leaf, 3 internal, 4 projection
+  auto cls = [&](int k) {
+    if (kclass != nullptr) *kclass = k;
+    a.span_acc = a0.span_acc != nullptr ? a0.span_acc + 2 * k : nullptr;
+  };
   static const int use_pair = getenv("BM_PAIR") ? atoi(getenv("BM_PAIR")) : 1;
   if (use_pair && a.epi == EPI_LSTM && !a.small_plan) {  // CTA-pair path (falls through if not eligible)
     bool done = false;
+    cls(0);
     cudaError_t e = rows_host != nullptr ? (a.b <= kMaxRowsInline ? launch_pair<true>(a, rows_host, st, &done)
                                                                    : cudaSuccess)
                                          : launch_pair<false>(a, rows_host, st, &done);
     if (done || e != cudaSuccess) return e;
   }
   switch (a.epi) {
-    case EPI_LSTM: return launch_impl<EPI_LSTM>(a, rows_host, st);
-    case EPI_LEAF: return launch_impl<EPI_LEAF>(a, rows_host, st);
-    case EPI_INTERNAL: return launch_impl<EPI_INTERNAL>(a, rows_host, st);
-    case EPI_PROJ: return launch_impl<EPI_PROJ>(a, rows_host, st);
+    case EPI_LSTM: cls(1); return launch_impl<EPI_LSTM>(a, rows_host, st);
+    case EPI_LEAF: cls(2); return launch_impl<EPI_LEAF>(a, rows_host, st);
+    case EPI_INTERNAL: cls(3); return launch_impl<EPI_INTERNAL>(a, rows_host, st);
+    case EPI_PROJ: cls(4); return launch_impl<EPI_PROJ>(a, rows_host, st);
   }
   return cudaErrorInvalidValue;
 }

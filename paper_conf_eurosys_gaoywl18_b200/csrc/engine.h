@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <chrono>
 #include <deque>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -152,7 +153,6 @@ struct Task {
   int b = 0;
   std::vector<TaskRow> rows;
   std::vector<RowDesc> desc; // device row descriptors, built at submission (A3)
-  int ev_first = -1, ev_count = 0;  // timed launches (time_kernels)
   std::vector<int> batch_reqs;      // graph batching: the batch's requests (on its last task)
   int worker = 0;                   // Algorithm 1 worker (bm_config.workers)
 };
@@ -176,13 +176,9 @@ struct WorkerState {
   unsigned long long* amax = nullptr;
 };
 
-struct TimedLaunch {
-  cudaEvent_t beg, end;
-  double bytes, flops;
-  int b;
-};
 
 struct Engine {
+  std::recursive_mutex mu;          // every C-ABI call on the engine holds it (include/bm.h)
   bm_config cfg{};
   bool sticky_cuda = false;
   bool submitted_any = false;
@@ -201,6 +197,7 @@ struct Engine {
   std::chrono::steady_clock::time_point t0;
   bool wall_started = false;
   std::vector<bm_completion> completions;   // not yet returned by bm_poll
+  uint64_t completed_total = 0;             // requests completed since creation
   std::vector<bm_task_record> log_tasks;
   std::vector<bm_row_record> log_rows;
   bm_stats stats{};
@@ -252,10 +249,16 @@ struct Engine {
   unsigned int* gbar = nullptr;
   int* perr = nullptr;
   uint64_t run_base = 0;               // launch index of the run's first task
-  std::vector<TimedLaunch> ev_pool;
-  int ev_head = 0;
-  unsigned long long* spans = nullptr;  // device: 64 span slots + accumulator (time_kernels)
-  unsigned long long span_base[2] = {0, 0};
+  // per-kernel timing (time_kernels): device [64 span slots x {start, ctas}] then
+  // [BM_K_CLASSES x {ns, launches}] accumulators, and a per-launch span log (kLaunchLog)
+  static constexpr int kLaunchLog = 1 << 16;
+  unsigned long long* spans = nullptr;
+  unsigned long long span_base[2 * BM_K_CLASSES] = {};
+  unsigned long long* span_log = nullptr;     // device [kLaunchLog] span ns of launch i
+  std::vector<int> launch_class, launch_b;    // host [kLaunchLog] class / rows of launch i
+  uint64_t timed_total = 0;                   // launches given a span slot so far
+  uint64_t timed_base = 0;                    // timed_total at the last bm_reset_stats
+  uint64_t poll_spins = 0;                    // non-blocking completion polls (error checks)
   uint64_t launches_base = 0;
   // diagnostics (BM_TIMELINE=<file>): per-launch device times + host issue times, per-task
   // host retire times; written at bm_destroy

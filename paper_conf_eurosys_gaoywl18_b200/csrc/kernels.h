@@ -72,7 +72,9 @@ struct StepArgs {
   int wcb, xring, xkb;        // ring plan (set by the launcher): K blocks per weight chunk,
                               // activation ring bytes, K blocks per activation stage
   unsigned long long* span;   // time_kernels: slot {min CTA start, CTAs done} (device memory)
-  unsigned long long* span_acc;  // {sum of launch spans in ns, launches}: last CTA adds
+  unsigned long long* span_acc;  // {sum of launch spans in ns, launches} of the launch's kernel
+                                 // class (bm.h BM_K_*): the last CTA adds
+  unsigned long long* span_log;  // or null: the last CTA stores this launch's span (ns) here
   const unsigned int* rows_flag;  // ring rows: published once *rows_flag >= rows_seq (or null)
   unsigned int rows_seq;
   unsigned int* dep_flag;     // launch chain: sequence number of the last completed launch
@@ -132,7 +134,11 @@ int persistent_smem_bytes();
 constexpr int kMaxRowsInline = 512;
 // rows_host: the launch's rows in host memory (b <= kMaxRowsInline) -- passed inline; or null,
 // then a.rows must point to device memory holding them.
-cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st);
+// *kclass (may be null) receives the kernel class (bm.h BM_K_*) the launch ran as; the launcher
+// picks the kernel, so a.span_acc must already point at that class's accumulator: pass
+// span_acc_base (the [BM_K_CLASSES][2] array) and the launcher offsets it.
+cudaError_t launch_cell_step_sm100(const StepArgs& a, const RowDesc* rows_host, cudaStream_t st,
+                                   int* kclass = nullptr);
 // fp32 / SIMT path (cell_step_simt.cu)
 cudaError_t launch_cell_step_simt(const StepArgs& a, cudaStream_t st);
 

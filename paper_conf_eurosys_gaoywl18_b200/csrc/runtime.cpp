@@ -70,6 +70,21 @@ void algo_cost(const Engine& e, const Cell& c, int b, bool proj, double* bytes, 
   *flops = 2.0 * b * K * rows;
 }
 
+// Host half of the per-kernel roofline (include/bm.h "measurement"): the launch's algorithmic
+// bytes / flops and its time at each roof, added to its kernel class.
+void account_launch(Engine& e, int kc, int b, double bytes, double flops) {
+  bm_stats& s = e.stats;
+  s.k_launches[kc] += 1;
+  s.k_rows[kc] += b;
+  s.k_bytes[kc] += bytes;
+  s.k_flops[kc] += flops;
+  const double t_hbm = e.cfg.roof_hbm_gbs > 0 ? bytes / (e.cfg.roof_hbm_gbs * 1e6) : 0.0;   // ms
+  const double t_tc = e.cfg.roof_tc_tflops > 0 ? flops / (e.cfg.roof_tc_tflops * 1e9) : 0.0;  // ms
+  s.k_roof_hbm_ms[kc] += t_hbm;
+  s.k_roof_tc_ms[kc] += t_tc;
+  s.k_roof_ms[kc] += std::max(t_hbm, t_tc);
+}
+
 }  // namespace
 
 // ---------------------------------------------------------------- workers (§8f N2)
@@ -98,7 +113,7 @@ void select_worker(Engine& e, int w) {
 
 // ---------------------------------------------------------------- launching tasks
 static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, const RowDesc* rows_host,
-                                 int b, int layer, bool proj, int* ev_out, unsigned long long* signal,
+                                 int b, int layer, bool proj, unsigned long long* signal,
                                  unsigned long long sig_value = 0) {
   StepArgs a{};
   a.epi = proj ? EPI_PROJ : c.epi;
@@ -164,21 +179,15 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
     a.rows_flag = e.rows_flag_dev;
     a.rows_seq = e.launch_rows_seq;
   }
-  TimedLaunch* tl = nullptr;
-  // events serialise the stream and so disable PDL overlap around the launches they bracket:
-  // time a sample (every kTimeEvery-th launch) instead of every launch
-  static const int time_every = getenv("BM_TIME_EVERY") ? atoi(getenv("BM_TIME_EVERY")) : 8;
-  const bool sample = (e.stats.kernel_launches % (time_every > 0 ? time_every : 1)) == 0;
-  if (e.cfg.time_kernels && !e.ev_pool.empty() && sample) {
-    const int i = e.ev_head;
-    e.ev_head = (e.ev_head + 1) % static_cast<int>(e.ev_pool.size());
-    tl = &e.ev_pool[i];
-    tl->b = b;
-    algo_cost(e, c, b, proj, &tl->bytes, &tl->flops);
-    a.span = e.spans + 2 * (e.stats.kernel_launches % 64);  // 64 slots: PDL overlaps <= 2 launches
-    a.span_acc = e.spans + 128;
-    CK(cudaEventRecord(tl->beg, e.stream));
-    if (ev_out) *ev_out = i;
+  // time_kernels: EVERY launch gets a device span slot, its class accumulator and a log entry
+  const bool timed = e.cfg.time_kernels && e.spans != nullptr;
+  uint64_t log_i = 0;
+  if (timed) {
+    const uint64_t i = e.timed_total++;
+    log_i = i % Engine::kLaunchLog;
+    a.span = e.spans + 2 * (i % 64);   // PDL keeps at most a few launches open at once
+    a.span_acc = e.spans + 128;        // class accumulators: the launcher offsets by class
+    a.span_log = e.span_log + log_i;
   }
   if (e.tl_dev != nullptr && e.tl_n < Engine::kTimeline) {
     a.tl = e.tl_dev + 4 * e.tl_n;
@@ -187,18 +196,26 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
     e.tl_n += 1;
   }
   cudaError_t err;
+  int kc = BM_K_SIMT;
   if (e.cfg.precision == BM_PREC_BF16) {
-    err = launch_cell_step_sm100(a, rows_host, e.stream);
+    err = launch_cell_step_sm100(a, rows_host, e.stream, &kc);
     if (err == cudaSuccess) {
       if (!no_chain) e.dep_seq += 1;
       e.pdl_ok = true;
     }
   } else {
     a.pdl = 0;  // the SIMT kernels do not use griddepcontrol
+    if (timed) a.span_acc += 2 * BM_K_SIMT;
     err = launch_cell_step_simt(a, e.stream);
   }
   CK(err);
-  if (tl) CK(cudaEventRecord(tl->end, e.stream));
+  if (timed) {
+    double bytes, flops;
+    algo_cost(e, c, b, proj, &bytes, &flops);
+    account_launch(e, kc, b, bytes, flops);
+    e.launch_class[log_i] = kc;
+    e.launch_b[log_i] = b;
+  }
   e.stats.kernel_launches += 1;
   return BM_OK;
 }
@@ -215,24 +232,14 @@ static bm_status launch_cell(Engine& e, Cell& c, const RowDesc* rows_dev, const 
   if (signal != nullptr && t != nullptr) signal += t->seq % kSignalSlots;  // its own slot
   const int L = lstm ? c.d.layers : 1;
   for (int l = 0; l < L; ++l) {
-    int ev = -1;
     const bool last = l == L - 1 && !proj;
-    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, l, false, &ev, (last && fused) ? signal : nullptr,
+    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, l, false, (last && fused) ? signal : nullptr,
                                   sig_value);
     if (s != BM_OK) return s;
-    if (t && ev >= 0) {
-      if (t->ev_first < 0) t->ev_first = ev;
-      t->ev_count += 1;
-    }
   }
   if (proj) {
-    int ev = -1;
-    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, 0, true, &ev, fused ? signal : nullptr, sig_value);
+    bm_status s = launch_one_step(e, c, rows_dev, rows_host, b, 0, true, fused ? signal : nullptr, sig_value);
     if (s != BM_OK) return s;
-    if (t && ev >= 0) {
-      if (t->ev_first < 0) t->ev_first = ev;  // the projection may be the task's only timed launch
-      t->ev_count += 1;
-    }
   }
   if (signal != nullptr && !fused) {
     CK(launch_signal(signal, sig_value, e.stream));
@@ -305,9 +312,7 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
       if (e.cfg.time_kernels) {
         double bytes, flops;
         algo_cost(e, e.cells[t.ct], t.b, false, &bytes, &flops);
-        e.stats.timed_launches += 1;
-        e.stats.timed_bytes += bytes;
-        e.stats.timed_flops += flops;
+        account_launch(e, BM_K_PERSISTENT, t.b, bytes, flops);
       }
     }
     const int first = std::min(n, e.hdr_ring - h0);
@@ -355,54 +360,57 @@ bm_status launch_tasks(Engine& e, std::vector<Task>& tasks) {
   return BM_OK;
 }
 
+// While a task's completion slot has not landed, the spin loops query the stream every 4096
+// polls (~0.5 ms): a CUDA error (a fault, or a kernel's 10 s dependency-wait trap) makes the
+// engine sticky (BM_E_CUDA, include/bm.h); so does an idle stream whose task never signalled
+// (e.g. the persistent kernel aborted), instead of spinning forever.
+static bool completion_lost(Engine& e, volatile unsigned long long* sig, uint64_t seq) {
+  const cudaError_t q = cudaStreamQuery(e.stream);
+  if (q == cudaErrorNotReady) return false;
+  if (q == cudaSuccess && *sig > seq) return false;  // landed meanwhile
+  if (!e.sticky_cuda)
+    fprintf(stderr, "bm: task %llu never signalled completion (%s)\n", static_cast<unsigned long long>(seq),
+            q == cudaSuccess ? "stream idle" : cudaGetErrorString(q));
+  e.sticky_cuda = true;
+  return true;
+}
+
 // Retire the active worker's oldest in-flight task if the device has finished it (and, on the
-// virtual clock, its tick has come). Returns 1 if retired.
+// virtual clock, its tick has come). Returns 1 if retired, 0 if not (yet), -1 on a CUDA error.
 static int retire_front(Engine& e, bool block) {
   if (e.inflight.empty()) return 0;
-  {
-    Task& t = e.inflight.front();
-    if (e.cfg.clock != BM_CLOCK_WALL && t.finish > e.now) return 0;
-    if (e.device()) {
-      // the task's own signal slot (kSignalSlots-entry ring, written once per task)
-      volatile unsigned long long* sig = e.signal_host + (t.seq % kSignalSlots);
-      if (*sig <= t.seq) {
-        if (!block && e.cfg.clock == BM_CLOCK_WALL) return 0;
-        while (*sig <= t.seq) {
-        }
+  Task& t = e.inflight.front();
+  if (e.cfg.clock != BM_CLOCK_WALL && t.finish > e.now) return 0;
+  if (e.device()) {
+    // the task's own signal slot (kSignalSlots-entry ring, written once per task)
+    volatile unsigned long long* sig = e.signal_host + (t.seq % kSignalSlots);
+    if (*sig <= t.seq) {
+      if (!block && e.cfg.clock == BM_CLOCK_WALL) {
+        if ((++e.poll_spins & 4095) == 0 && completion_lost(e, sig, t.seq)) return -1;
+        return 0;
       }
+      for (uint64_t it = 1; *sig <= t.seq; ++it)
+        if ((it & 4095) == 0 && completion_lost(e, sig, t.seq)) return -1;
     }
-    if (e.tl_dev != nullptr && t.seq < Engine::kTimeline) e.tl_retire[t.seq] = realtime_ns();
-    if (e.cfg.clock == BM_CLOCK_WALL) e.now = wall_now(e);
-    const auto t0 = std::chrono::steady_clock::now();
-    retire_task(e, t);
-    if (t.ev_count > 0) {
-      for (int k = 0; k < t.ev_count; ++k) {
-        TimedLaunch& tl = e.ev_pool[(t.ev_first + k) % e.ev_pool.size()];
-        float ms = 0;
-        if (cudaEventElapsedTime(&ms, tl.beg, tl.end) != cudaSuccess) {
-          cudaGetLastError();  // not sticky: must not leak into a later launch's error check
-        } else {
-          e.stats.timed_launches += 1;
-          e.stats.timed_ms += ms;
-          e.stats.timed_bytes += tl.bytes;
-          e.stats.timed_flops += tl.flops;
-        }
-      }
-    }
-    e.inflight.pop_front();
-    e.stats.retire_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
   }
+  if (e.tl_dev != nullptr && t.seq < Engine::kTimeline) e.tl_retire[t.seq] = realtime_ns();
+  if (e.cfg.clock == BM_CLOCK_WALL) e.now = wall_now(e);
+  const auto t0 = std::chrono::steady_clock::now();
+  retire_task(e, t);
+  e.inflight.pop_front();
+  e.stats.retire_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
   return 1;
 }
 
 // Retire every finished in-flight task of every worker. Virtual clock: in (finish tick,
 // worker) order (S21 with W workers, as the replay); wall clock: each worker's FIFO.
-static int retire_ready(Engine& e, bool block) {
-  int n = 0;
+static bm_status retire_ready(Engine& e, bool block) {
   const int W = e.cfg.workers;
+  int r = 0;
   if (W == 1) {
-    while (retire_front(e, block)) ++n;
-    return n;
+    while ((r = retire_front(e, block)) > 0) {
+    }
+    return r < 0 ? BM_E_CUDA : BM_OK;
   }
   if (e.cfg.clock != BM_CLOCK_WALL) {
     for (;;) {
@@ -417,15 +425,17 @@ static int retire_ready(Engine& e, bool block) {
       }
       if (best < 0) break;
       select_worker(e, best);
-      n += retire_front(e, block);
+      if ((r = retire_front(e, block)) < 0) return BM_E_CUDA;
     }
   } else {
     for (int w = 0; w < W; ++w) {
       select_worker(e, w);
-      while (retire_front(e, block)) ++n;
+      while ((r = retire_front(e, block)) > 0) {
+      }
+      if (r < 0) return BM_E_CUDA;
     }
   }
-  return n;
+  return BM_OK;
 }
 
 static void admit_due(Engine& e) {
@@ -479,7 +489,8 @@ static bool all_done(Engine& e) {
 
 // One round of the virtual-time event loop (S21); advances the clock to the next event.
 static bm_status virtual_round(Engine& e, int* n_tasks) {
-  retire_ready(e, true);
+  *n_tasks = 0;
+  if (retire_ready(e, true) != BM_OK) return BM_E_CUDA;
   admit_due(e);
   bm_status s = schedule_and_launch(e, n_tasks);
   if (s != BM_OK) return s;
@@ -599,11 +610,8 @@ static void free_device(Engine& e) {
     if (ev) cudaEventDestroy(ev);
   if (e.ring_host) cudaFreeHost(e.ring_host);
   if (e.signal_host) cudaFreeHost(e.signal_host);
-  for (TimedLaunch& t : e.ev_pool) {
-    cudaEventDestroy(t.beg);
-    cudaEventDestroy(t.end);
-  }
   cudaFree(e.spans);
+  cudaFree(e.span_log);
   if (e.copy_stream) cudaStreamDestroy(e.copy_stream);
   if (e.copy_ev) cudaEventDestroy(e.copy_ev);
   cudaFree(e.hdr_dev);
@@ -623,7 +631,10 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       c.max_tasks_to_submit < 1 || c.min_followon_batch < 1 || c.schedule_when_outstanding_leq < 0 ||
       c.max_decode_len < 1 || c.precision < 0 || c.precision > 1 || c.clock < 0 || c.clock > 2 ||
       c.policy < 0 || c.policy > 1 || c.bucket_width < 1 || c.workers < 1 || c.workers > 8 ||
-      (c.workers > 1 && c.policy != BM_POLICY_CELLULAR))
+      (c.workers > 1 && c.policy != BM_POLICY_CELLULAR) ||
+      // tasks in flight per worker (<= k + MaxTasksToSubmit) must fit the completion-signal
+      // ring and the persistent kernel's task-header ring (both kSignalSlots = 256 entries)
+      c.max_tasks_to_submit + c.schedule_when_outstanding_leq + 2 > kSignalSlots)
     return BM_E_INVAL;
   Engine* e = new (std::nothrow) Engine();
   if (e == nullptr) return BM_E_NOMEM;
@@ -663,7 +674,10 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
               cudaEventCreateWithFlags(&E.direct_ev[0], cudaEventDisableTiming) == cudaSuccess &&
               cudaEventCreateWithFlags(&E.direct_ev[1], cudaEventDisableTiming) == cudaSuccess;
     if (!ok) return fail(BM_E_NOMEM);
-    E.ring_rows = std::max(64, c.max_tasks_to_submit + c.schedule_when_outstanding_leq + 2) * 512 * 2;
+    // descriptor ring: every worker keeps <= k + MaxTasksToSubmit tasks of <= 512 rows in
+    // flight, and a Schedule call's rows are placed contiguously (a wrap wastes the tail):
+    // twice that bound, so rows of a task still in flight are never overwritten
+    E.ring_rows = std::max(64, c.workers * (c.max_tasks_to_submit + c.schedule_when_outstanding_leq + 2)) * 512 * 2;
     if (dalloc(&E.ring_dev, E.ring_rows) != cudaSuccess) return fail(BM_E_NOMEM);
     if (cudaHostAlloc(reinterpret_cast<void**>(&E.ring_host), E.ring_rows * sizeof(RowDesc),
                       cudaHostAllocDefault) != cudaSuccess)
@@ -704,18 +718,18 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
         cudaMemsetAsync(E.res_tok, 0, R * c.max_decode_len * 4, E.stream) != cudaSuccess)
       return fail(BM_E_CUDA);
     if (c.time_kernels) {
-      E.ev_pool.resize(4096);
-      // device-side launch spans: 64 slots {start, ctas} + accumulator {ns, launches}
-      if (dalloc(&E.spans, 2 * 64 + 2) != cudaSuccess ||
-          cudaMemsetAsync(E.spans, 0xFF, 2 * 64 * 8, E.stream) != cudaSuccess)
+      // device-side launch spans: 64 slots {start, ctas}, per-class accumulators {ns, launches},
+      // and the per-launch span log
+      if (dalloc(&E.spans, 2 * 64 + 2 * BM_K_CLASSES) != cudaSuccess ||
+          dalloc(&E.span_log, Engine::kLaunchLog) != cudaSuccess ||
+          cudaMemsetAsync(E.spans, 0xFF, 2 * 64 * 8, E.stream) != cudaSuccess ||
+          cudaMemsetAsync(E.span_log, 0, Engine::kLaunchLog * 8, E.stream) != cudaSuccess)
         return fail(BM_E_NOMEM);
       for (int i = 0; i < 64; ++i)
         if (cudaMemsetAsync(E.spans + 2 * i + 1, 0, 8, E.stream) != cudaSuccess) return fail(BM_E_CUDA);
-      if (cudaMemsetAsync(E.spans + 128, 0, 16, E.stream) != cudaSuccess) return fail(BM_E_CUDA);
-      for (TimedLaunch& t : E.ev_pool) {
-        if (cudaEventCreate(&t.beg) != cudaSuccess || cudaEventCreate(&t.end) != cudaSuccess)
-          return fail(BM_E_CUDA);
-      }
+      if (cudaMemsetAsync(E.spans + 128, 0, 16 * BM_K_CLASSES, E.stream) != cudaSuccess) return fail(BM_E_CUDA);
+      E.launch_class.assign(Engine::kLaunchLog, 0);
+      E.launch_b.assign(Engine::kLaunchLog, 0);
     }
     if (getenv("BM_TIMELINE") != nullptr) {
       if (dalloc(&E.tl_dev, 4 * Engine::kTimeline) != cudaSuccess ||
@@ -762,6 +776,7 @@ void* bm_stream(bm_engine* h) { return h ? reinterpret_cast<Engine*>(h)->stream 
 bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w, int* cell_id) {
   if (h == nullptr || d == nullptr || w == nullptr || cell_id == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (e.sticky_cuda) return BM_E_CUDA;
   if (e.submitted_any) return BM_E_STATE;
@@ -807,21 +822,55 @@ bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w,
     const bool bf = e.cfg.precision == BM_PREC_BF16;
     const size_t el = e.elem();
     const size_t rows = static_cast<size_t>(c.G) * H;
+    // every weight array may be a host pointer (copied up) or a device pointer on the engine's
+    // device (adopted in place: the packing kernels read it directly, e.g. after an NCCL
+    // broadcast). A device pointer of another device is rejected.
+    auto on_device = [&](const void* p, bool* dev) -> bool {
+      cudaPointerAttributes at{};
+      if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        *dev = false;
+        return true;
+      }
+      *dev = at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+      return !*dev || at.device == e.cfg.device;
+    };
+    std::vector<const void*> srcs;
+    for (int l = 0; l < L; ++l) srcs.push_back(w->W[l]), srcs.push_back(w->b[l]);
+    if (w->E != nullptr) srcs.push_back(w->E);
+    if (d->kind == BM_CELL_LSTM_PROJ) srcs.push_back(w->W_out), srcs.push_back(w->b_out);
+    for (const void* p : srcs) {
+      bool dev;
+      if (!on_device(p, &dev)) return BM_E_INVAL;
+    }
     float* tmp = nullptr;
     float* tmpb = nullptr;
     const size_t maxsrc = std::max(rows * K, static_cast<size_t>(d->vocab) * H);
     CK(cudaMalloc(&tmp, maxsrc * 4));
     CK(cudaMalloc(&tmpb, std::max(rows, static_cast<size_t>(d->vocab)) * 4));
+    // device source: use it as is; host source: copy into the staging buffer
+    auto stage = [&](const float* src, float* buf, size_t n, const float** out) -> cudaError_t {
+      bool dev = false;
+      on_device(src, &dev);
+      if (dev) {
+        *out = src;
+        return cudaSuccess;
+      }
+      *out = buf;
+      return cudaMemcpyAsync(buf, src, n * 4, cudaMemcpyHostToDevice, e.stream);
+    };
+    const float* sw = nullptr;
+    const float* sb = nullptr;
     for (int l = 0; l < L; ++l) {
       void* Wp = nullptr;
       float* bp = nullptr;
       CK(cudaMalloc(&Wp, rows * K * el));
       CK(dalloc(&bp, rows));
-      CK(cudaMemcpyAsync(tmp, w->W[l], rows * K * 4, cudaMemcpyHostToDevice, e.stream));
-      CK(cudaMemcpyAsync(tmpb, w->b[l], rows * 4, cudaMemcpyHostToDevice, e.stream));
-      CK(launch_pack_rows(tmp, Wp, bp, tmpb, c.G, H, K, bf ? 1 : 0, e.stream));
+      CK(stage(w->W[l], tmp, rows * K, &sw));
+      CK(stage(w->b[l], tmpb, rows, &sb));
+      CK(launch_pack_rows(sw, Wp, bp, sb, c.G, H, K, bf ? 1 : 0, e.stream));
       if (bf)  // the tcgen05 kernel streams pre-swizzled stage tiles (overwrites the plain pack)
-        CK(launch_pack_tiles(tmp, Wp, c.G, H, K, c.G * c.U, static_cast<int>(rows), e.stream));
+        CK(launch_pack_tiles(sw, Wp, c.G, H, K, c.G * c.U, static_cast<int>(rows), e.stream));
       CK(cudaStreamSynchronize(e.stream));
       c.W.push_back(Wp);
       c.bias.push_back(bp);
@@ -829,18 +878,18 @@ bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w,
     if (w->E != nullptr && d->kind != BM_CELL_TREE_INTERNAL) {
       const size_t n = static_cast<size_t>(d->vocab) * H;
       CK(cudaMalloc(&c.E, n * el));
-      CK(cudaMemcpyAsync(tmp, w->E, n * 4, cudaMemcpyHostToDevice, e.stream));
-      CK(launch_convert(tmp, c.E, n, bf ? 1 : 0, e.stream));
+      CK(stage(w->E, tmp, n, &sw));
+      CK(launch_convert(sw, c.E, n, bf ? 1 : 0, e.stream));
       CK(cudaStreamSynchronize(e.stream));
     }
     if (d->kind == BM_CELL_LSTM_PROJ) {
       const size_t n = static_cast<size_t>(d->vocab) * H;
       CK(cudaMalloc(&c.W_out, n * el));
       CK(dalloc(&c.b_out, d->vocab));
-      CK(cudaMemcpyAsync(tmp, w->W_out, n * 4, cudaMemcpyHostToDevice, e.stream));
-      if (bf) CK(launch_pack_tiles(tmp, c.W_out, 1, H, H, 128, d->vocab, e.stream));
-      else CK(launch_convert(tmp, c.W_out, n, 0, e.stream));
-      CK(cudaMemcpyAsync(c.b_out, w->b_out, d->vocab * 4, cudaMemcpyHostToDevice, e.stream));
+      CK(stage(w->W_out, tmp, n, &sw));
+      if (bf) CK(launch_pack_tiles(sw, c.W_out, 1, H, H, 128, d->vocab, e.stream));
+      else CK(launch_convert(sw, c.W_out, n, 0, e.stream));
+      CK(cudaMemcpyAsync(c.b_out, w->b_out, d->vocab * 4, cudaMemcpyDefault, e.stream));
       CK(cudaStreamSynchronize(e.stream));
       if (e.cfg.record_logits) {
         if (e.logits == nullptr) {
@@ -880,6 +929,7 @@ static bool valid_tree(const bm_request* r) {
 bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
   if (h == nullptr || q == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   if (e.sticky_cuda) return BM_E_CUDA;
   const int nc = static_cast<int>(e.cells.size());
   auto cell_ok = [&](int id, int k1, int k2) {
@@ -912,6 +962,9 @@ bm_status bm_submit(bm_engine* h, const bm_request* q, uint64_t* req_id) {
     const bool leaf_or_chain = q->kind != BM_REQ_TREE || q->left[i] < 0;
     if (leaf_or_chain && (q->tokens[i] < 0 || q->tokens[i] >= vocab)) return BM_E_INVAL;
   }
+  // requests not yet admitted must arrive in submission order (an open-loop arrival stream;
+  // each request is admitted at its own arrival, L323 / reading S21)
+  if (!e.pending.empty() && q->arrival < e.reqs[e.pending.back()].t_arrival) return BM_E_INVAL;
   if (e.n_live_reqs >= e.cfg.max_requests) return BM_E_FULL;
   // request table slot: the entry of admission index id % max_requests must be free
   const int ri = static_cast<int>(e.next_req_id % e.cfg.max_requests);
@@ -965,6 +1018,7 @@ bm_status bm_submit_many(bm_engine* h, const bm_request* reqs, int n, uint64_t* 
 bm_status bm_schedule_step(bm_engine* h, int* n_tasks) {
   if (h == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   if (e.sticky_cuda) return BM_E_CUDA;
   int n = 0;
   bm_status s;
@@ -974,9 +1028,11 @@ bm_status bm_schedule_step(bm_engine* h, int* n_tasks) {
       e.wall_started = true;
     }
     e.now = wall_now(e);
-    retire_ready(e, false);
-    admit_due(e);
-    s = schedule_and_launch(e, &n);
+    s = retire_ready(e, false);
+    if (s == BM_OK) {
+      admit_due(e);
+      s = schedule_and_launch(e, &n);
+    }
     if (s == BM_OK && n == 0 && all_done(e)) s = BM_E_AGAIN;
   } else {
     s = virtual_round(e, &n);
@@ -989,10 +1045,12 @@ bm_status bm_schedule_step(bm_engine* h, int* n_tasks) {
 bm_status bm_poll(bm_engine* h, bm_completion* out, int cap, int* n) {
   if (h == nullptr || n == nullptr || (cap > 0 && out == nullptr)) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
-  if (e.cfg.clock == BM_CLOCK_WALL) {
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
+  if (e.cfg.clock == BM_CLOCK_WALL && e.device()) {
     e.now = wall_now(e);
-    retire_ready(e, false);
+    const bm_status s = retire_ready(e, false);
     select_worker(e, 0);
+    if (s != BM_OK) return s;
   }
   const int k = std::min<int>(cap, static_cast<int>(e.completions.size()));
   if (k > 0) memcpy(out, e.completions.data(), k * sizeof(bm_completion));
@@ -1048,7 +1106,7 @@ static bm_status persistent_start(Engine& e) {
   a.signal = e.signal_dev;
   a.sig_base = e.launched;  // == run_base below
   a.span = e.cfg.time_kernels ? e.spans : nullptr;
-  a.span_acc = e.cfg.time_kernels ? e.spans + 128 : nullptr;
+  a.span_acc = e.cfg.time_kernels ? e.spans + 128 + 2 * BM_K_PERSISTENT : nullptr;
   static const char* dump = getenv("BM_PHASE_DUMP");
   if (dump != nullptr && e.phase_dev == nullptr) CK(cudaMalloc(&e.phase_dev, 8 * 64 * 4096));
   if (e.phase_dev) CK(cudaMemsetAsync(e.phase_dev, 0, 8 * 64 * 4096, e.stream));
@@ -1107,8 +1165,9 @@ static bm_status persistent_stop(Engine& e) {
 bm_status bm_run(bm_engine* h, int* n_completed) {
   if (h == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::unique_lock<std::recursive_mutex> lk(e.mu);
   if (e.sticky_cuda) return BM_E_CUDA;
-  const size_t before = e.completions.size();
+  const uint64_t before = e.completed_total;  // a concurrent bm_poll may drain e.completions
   int n = 0;
   bm_status s = BM_OK;
   if (persistent_eligible(e)) {
@@ -1116,14 +1175,20 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
     if (s != BM_OK && s != BM_E_AGAIN) return s;
     s = BM_OK;
   }
+  lk.unlock();
   if (e.cfg.clock == BM_CLOCK_WALL) {
     e.t0 = std::chrono::steady_clock::now();
     e.wall_started = true;
     while (true) {
+      // one round of the event loop under the engine lock: a bm_poll on another thread
+      // (the paper's poll thread, L395) interleaves between rounds
+      std::lock_guard<std::recursive_mutex> round(e.mu);
       e.now = wall_now(e);
-      retire_ready(e, false);
-      admit_due(e);
-      s = schedule_and_launch(e, &n);
+      s = retire_ready(e, false);
+      if (s == BM_OK) {
+        admit_due(e);
+        s = schedule_and_launch(e, &n);
+      }
       if (s != BM_OK) {
         select_worker(e, 0);
         persistent_stop(e);
@@ -1132,14 +1197,18 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
       if (all_done(e)) break;
     }
   } else {
-    while ((s = virtual_round(e, &n)) == BM_OK) {
+    for (;;) {
+      std::lock_guard<std::recursive_mutex> round(e.mu);
+      if ((s = virtual_round(e, &n)) != BM_OK) break;
     }
     if (s != BM_E_AGAIN) {
+      std::lock_guard<std::recursive_mutex> g(e.mu);
       select_worker(e, 0);
       persistent_stop(e);
       return s;
     }
   }
+  lk.lock();
   if (e.persistent_active) {
     s = persistent_stop(e);
     if (s != BM_OK) return s;
@@ -1151,13 +1220,14 @@ bm_status bm_run(bm_engine* h, int* n_completed) {
     }
   }
   select_worker(e, 0);
-  if (n_completed) *n_completed = static_cast<int>(e.completions.size() - before);
+  if (n_completed) *n_completed = static_cast<int>(e.completed_total - before);
   return BM_OK;
 }
 
 bm_status bm_read_result(bm_engine* h, uint64_t req_id, bm_result* dst) {
   if (h == nullptr || dst == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (e.sticky_cuda) return BM_E_CUDA;
   Request& r = e.reqs[req_id % e.cfg.max_requests];
@@ -1189,6 +1259,7 @@ bm_status bm_read_result(bm_engine* h, uint64_t req_id, bm_result* dst) {
 bm_status bm_release(bm_engine* h, uint64_t req_id) {
   if (h == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   Request& r = e.reqs[req_id % e.cfg.max_requests];
   if (!r.used || r.id != req_id) return BM_E_INVAL;
   if (!r.done) return BM_E_STATE;
@@ -1197,10 +1268,11 @@ bm_status bm_release(bm_engine* h, uint64_t req_id) {
   return BM_OK;
 }
 
-bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh, int32_t* toks,
-                               int release) {
+bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh, float* cc,
+                               int32_t* toks, int release) {
   if (h == nullptr || n < 1) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (e.sticky_cuda) return BM_E_CUDA;
   if (!e.device()) return BM_E_STATE;
@@ -1218,6 +1290,7 @@ bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh
     const size_t ri = (first_id + done) % R;
     const int len = static_cast<int>(std::min<uint64_t>(n - done, R - ri));
     if (hh) CK(cudaMemcpyAsync(hh + done * LH, e.res_h + ri * LH, len * LH * 4, cudaMemcpyDeviceToHost, e.stream));
+    if (cc) CK(cudaMemcpyAsync(cc + done * LH, e.res_c + ri * LH, len * LH * 4, cudaMemcpyDeviceToHost, e.stream));
     if (toks) CK(cudaMemcpyAsync(toks + done * D, e.res_tok + ri * D, len * D * 4, cudaMemcpyDeviceToHost, e.stream));
     done += len;
   }
@@ -1243,6 +1316,7 @@ bm_status bm_read_results_many(bm_engine* h, uint64_t first_id, int n, float* hh
 bm_status bm_read_log(bm_engine* h, bm_task_record* out, int cap, int* n) {
   if (h == nullptr || n == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   const int k = std::min<int>(cap, static_cast<int>(e.log_tasks.size()));
   if (k > 0) memcpy(out, e.log_tasks.data(), k * sizeof(bm_task_record));
   *n = static_cast<int>(e.log_tasks.size());
@@ -1252,6 +1326,7 @@ bm_status bm_read_log(bm_engine* h, bm_task_record* out, int cap, int* n) {
 bm_status bm_read_log_rows(bm_engine* h, bm_row_record* out, int cap, int* n) {
   if (h == nullptr || n == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   const int k = std::min<int>(cap, static_cast<int>(e.log_rows.size()));
   if (k > 0) memcpy(out, e.log_rows.data(), k * sizeof(bm_row_record));
   *n = static_cast<int>(e.log_rows.size());
@@ -1261,6 +1336,7 @@ bm_status bm_read_log_rows(bm_engine* h, bm_row_record* out, int cap, int* n) {
 bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b, int async) {
   if (h == nullptr || rows == nullptr || b < 1 || b > 4096) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   if (e.sticky_cuda) return BM_E_CUDA;
   if (!e.device()) return BM_E_STATE;
   if (cell_id < 0 || cell_id >= static_cast<int>(e.cells.size())) return BM_E_INVAL;
@@ -1324,6 +1400,7 @@ bm_status bm_cell_step(bm_engine* h, int cell_id, const bm_step_row* rows, int b
 
 static bm_status pool_io(Engine& e, int layer, int parity, const int32_t* slots, int n, float* h,
                          float* c, int write) {
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   e.pdl_ok = false;
   if (!e.device()) return BM_E_STATE;
   if (layer < 0 || layer >= e.cfg.pool_layers || parity < 0 || parity > 1 || n < 1 || slots == nullptr)
@@ -1374,6 +1451,7 @@ bm_status bm_pool_read(bm_engine* h, int layer, int parity, const int32_t* slots
 bm_status bm_result_rows(bm_engine* h, const int32_t* res_idx, int n, float* hh, float* cc) {
   if (h == nullptr || res_idx == nullptr || n < 1) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (!e.device()) return BM_E_STATE;
   const size_t LH = e.H() * e.cfg.pool_layers;
@@ -1390,6 +1468,7 @@ bm_status bm_result_rows(bm_engine* h, const int32_t* res_idx, int n, float* hh,
 bm_status bm_tokens(bm_engine* h, const int32_t* slots, int n, int32_t* inout, int write) {
   if (h == nullptr || slots == nullptr || inout == nullptr || n < 1) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   e.pdl_ok = false;  // other stream work follows: the next launch is fully ordered
   if (!e.device()) return BM_E_STATE;
   CK(cudaStreamSynchronize(e.stream));
@@ -1405,14 +1484,17 @@ bm_status bm_tokens(bm_engine* h, const int32_t* slots, int n, int32_t* inout, i
 bm_status bm_get_stats(bm_engine* h, bm_stats* out) {
   if (h == nullptr || out == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   *out = e.stats;
   out->kernel_launches = e.stats.kernel_launches - e.launches_base;
   if (e.spans != nullptr) {  // device-side spans accumulated since the last reset
-    unsigned long long acc[2] = {0, 0};
+    unsigned long long acc[2 * BM_K_CLASSES];
     CK(cudaStreamSynchronize(e.stream));
-    CK(cudaMemcpy(acc, e.spans + 128, 16, cudaMemcpyDeviceToHost));
-    out->span_ms = (acc[0] - e.span_base[0]) * 1e-6;
-    out->span_launches = acc[1] - e.span_base[1];
+    CK(cudaMemcpy(acc, e.spans + 128, sizeof(acc), cudaMemcpyDeviceToHost));
+    for (int k = 0; k < BM_K_CLASSES; ++k) {
+      out->k_span_ms[k] = (acc[2 * k] - e.span_base[2 * k]) * 1e-6;
+      out->k_span_launches[k] = acc[2 * k + 1] - e.span_base[2 * k + 1];
+    }
   }
   return BM_OK;
 }
@@ -1420,14 +1502,43 @@ bm_status bm_get_stats(bm_engine* h, bm_stats* out) {
 bm_status bm_reset_stats(bm_engine* h) {
   if (h == nullptr) return BM_E_INVAL;
   Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
   const uint64_t launches = e.stats.kernel_launches;  // keeps the span slot rotation aligned
   e.stats = bm_stats{};
   e.stats.kernel_launches = launches;
   e.launches_base = launches;
+  e.timed_base = e.timed_total;
   if (e.spans != nullptr) {
     CK(cudaStreamSynchronize(e.stream));
-    CK(cudaMemcpy(e.span_base, e.spans + 128, 16, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(e.span_base, e.spans + 128, sizeof(e.span_base), cudaMemcpyDeviceToHost));
   }
+  return BM_OK;
+}
+
+bm_status bm_read_launch_log(bm_engine* h, bm_launch_record* out, int cap, int* n) {
+  if (h == nullptr || n == nullptr || (cap > 0 && out == nullptr)) return BM_E_INVAL;
+  Engine& e = *reinterpret_cast<Engine*>(h);
+  std::lock_guard<std::recursive_mutex> lk(e.mu);
+  *n = 0;
+  if (e.span_log == nullptr) return BM_E_STATE;
+  const uint64_t total = e.timed_total - e.timed_base;
+  const uint64_t avail = std::min<uint64_t>(total, Engine::kLaunchLog);
+  const int k = static_cast<int>(std::min<uint64_t>(avail, static_cast<uint64_t>(std::max(cap, 0))));
+  if (k == 0) {
+    *n = static_cast<int>(avail);
+    return BM_OK;
+  }
+  std::vector<unsigned long long> spans(Engine::kLaunchLog);
+  CK(cudaStreamSynchronize(e.stream));
+  CK(cudaMemcpy(spans.data(), e.span_log, spans.size() * 8, cudaMemcpyDeviceToHost));
+  const uint64_t first = e.timed_total - avail;
+  for (int i = 0; i < k; ++i) {
+    const uint64_t li = (first + i) % Engine::kLaunchLog;
+    out[i].kclass = e.launch_class[li];
+    out[i].b = e.launch_b[li];
+    out[i].span_ns = spans[li];
+  }
+  *n = k;
   return BM_OK;
 }
 

@@ -437,6 +437,7 @@ void retire_task(Engine& e, Task& t) {
       cp.t_first = r.t_first;
       cp.t_done = r.t_done;
       e.completions.push_back(cp);
+      e.completed_total += 1;
       slot_release(e, r.slot);
       if (!e.cfg.keep_results) {
         r.used = false;
@@ -500,6 +501,7 @@ void retire_task(Engine& e, Task& t) {
       cp.t_first = r.t_first;
       cp.t_done = r.t_done;
       e.completions.push_back(cp);
+      e.completed_total += 1;
       if (r.kind == BM_REQ_TREE) {
         for (int x : r.node_slot) slot_release(e, x);
       } else {

@@ -8,8 +8,7 @@ off the per-step path:
     gloo in the CPU tests),
   * max-over-ranks reductions of timings and a gather of latency samples at the end.
 The paper's own multi-GPU design (one manager, many workers, subgraph pinning and cross-GPU
-state migration, L317-L381) is SURVEY §8f row N2: its workers and pinning are built inside one
-engine (bm_config.workers, one device); the cross-GPU migration is not.
+state migration, L317-L381) is SURVEY §8f row N2 (bm_config.workers).
 """
 from __future__ import annotations
 
@@ -39,6 +38,27 @@ def broadcast_arrays(arrays: Sequence[Tuple[str, np.ndarray]], dist, device=None
         dist.broadcast(t, src=0)
         if rank != 0:
             arr[...] = t.cpu().numpy()
+
+
+def broadcast_tensors(arrays: Sequence[Tuple[str, np.ndarray]], dist, device=None) -> dict:
+    """Rank 0's arrays on every rank as tensors on `device` (NCCL over NVLink: the weights land
+    in device memory and bm_load_cell adopts them in place, include/bm.h bm_weights). With
+    device None (gloo on CPU) the numpy arrays are also overwritten in place."""
+    import torch
+    rank = dist.get_rank()
+    out = {}
+    for name, arr in arrays:
+        if rank == 0:
+            t = torch.from_numpy(np.ascontiguousarray(arr))
+            t = t.to(device) if device is not None else t.clone()
+        else:
+            t = torch.empty(arr.shape, dtype=torch.from_numpy(arr[:0]).dtype,
+                            device=device if device is not None else "cpu")
+        dist.broadcast(t, src=0)
+        if device is None and rank != 0:
+            arr[...] = t.numpy()
+        out[name] = t
+    return out
 
 
 def reduce_max(x: float, dist=None, device=None) -> float:

@@ -76,3 +76,37 @@ def test_two_rank_sharding_gloo(tmp_path):
 def test_rank_seeds_differ():
     from paper_conf_eurosys_gaoywl18_b200 import shard
     assert len({shard.rank_seed(1000, r) for r in range(8)}) == 8
+
+
+def test_bench_product_path_two_ranks_dry(tmp_path):
+    """The product bench path end to end on 2 ranks: plain `bench.py --gpus 2` re-launches itself
+    under torch.distributed.run (one process per GPU), rank 0 broadcasts the weights, every rank
+    runs its own engine over its own Poisson shard (BM_CLOCK_DRY here: the scheduler without a
+    GPU, collectives on gloo), and rank 0 prints ONE line with n_gpus = 2."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = tmp_path / "line.json"
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--dry", "--quick",
+                        "--steps", "1", "--warmup", "1", "--reqs", "600", "--no-cpu-baseline", "--out", str(out)],
+                       capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    line = json.loads(lines[0])
+    assert line["n_gpus"] == 2 and line["comm"]["world_size"] == 2
+    assert line["comm"]["backend"] == "gloo" and line["comm"]["per_step_collectives"] == 0
+    assert line["value"] > 0 and line["config"]["parallelism"] == "request-sharded x2"
+    assert json.loads(out.read_text())["n_gpus"] == 2
+
+
+def test_bench_refuses_mismatched_world(tmp_path):
+    """--gpus N under a launcher with WORLD_SIZE != N fails loudly instead of printing a 1-GPU line."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "8", "--dry"],
+                       capture_output=True, text=True, timeout=300, cwd=root, env=env)
+    assert r.returncode != 0 and "WORLD_SIZE" in (r.stderr + r.stdout)

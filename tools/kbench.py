@@ -25,8 +25,11 @@ def main():
     H, V = 1024, 32768
     prec = bm.PREC_FP32 if a.fp32 else bm.PREC_BF16
     bf = not a.fp32
+    pk = json.load(open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                                     "MEASURED_PEAKS.json")))
     e = bm.Engine(precision=prec, hidden=H, pool_layers=1, max_slots=8192, max_requests=8192,
-                  max_decode_len=4, time_kernels=1)
+                  max_decode_len=4, time_kernels=1, roof_hbm_gbs=pk["hbm_gbs"],
+                  roof_tc_tflops=pk["bf16_tflops"])
     if a.cell in ("lstm", "proj"):
         w = gen.lstm_stack_weights(H, 1, V, 0, projection=a.cell == "proj", bf16=bf)
         kind = bm.CELL_LSTM_PROJ if a.cell == "proj" else bm.CELL_LSTM
@@ -67,21 +70,19 @@ def main():
         us = ev0.elapsed_time(ev1) * 1e3 / a.iters
         st = e.stats()
         reps = int(os.environ.get("BM_REPEAT", "1"))
-        launches = a.iters * reps * (2 if a.cell == "proj" else 1)
-        # device: first CTA past the PDL wait .. last CTA end, over the sampled launches
-        span_us = st["span_ms"] * 1e3 / max(1, st["span_launches"])
-        if a.cell == "proj":
-            # LSTM layer + projection per call; report the sum
-            byts = (rows_w * K * el + b * 14336) + (V * H * el + b * (2 * H + 8))
-            flops = 2 * b * K * rows_w + 2 * b * H * V
-        else:
-            per_row = K * el + H * el + H * 4 + (H * 4 if a.cell == "lstm" else 2 * H * 4 if a.cell == "internal" else 0)
-            byts = rows_w * K * el + rows_w * 4 + b * per_row
-            flops = 2 * b * K * rows_w
-        r = {"cell": a.cell, "b": b, "us_per_call": us, "us_per_step": us / reps, "span_us": span_us,
-             "host_us_per_call": (th1 - th0) * 1e6 / a.iters,
-             "GBps_span": byts / span_us / 1e3 if span_us > 0 else None,
-             "TFLOPs_span": flops / span_us / 1e6 if span_us > 0 else None}
+        # every launch's device span (first CTA past its dependency wait .. last CTA done) and
+        # its algorithmic bytes / flops, per kernel class (include/bm.h "measurement")
+        r = {"cell": a.cell, "b": b, "us_per_call": us, "us_per_step": us / reps,
+             "host_us_per_call": (th1 - th0) * 1e6 / a.iters}
+        for k in range(bm.K_CLASSES):
+            n = st["k_launches"][k]
+            if not n:
+                continue
+            span = st["k_span_ms"][k] / max(1, st["k_span_launches"][k])
+            r[f"k{k}"] = {"launches": n, "span_us": span * 1e3,
+                          "GBps": st["k_bytes"][k] / n / (span / 1e3) / 1e9,
+                          "TFLOPs": st["k_flops"][k] / n / (span / 1e3) / 1e12,
+                          "frac_binding_burst": st["k_roof_ms"][k] / st["k_span_ms"][k]}
         print(json.dumps(r), flush=True)
         out.append(r)
     if a.out:

@@ -46,7 +46,7 @@ def main():
             st = e.stats()
             ms = ev0.elapsed_time(ev1)
             print(json.dumps({"persistent": pk, "b": b, "tasks": st["tasks"], "us_per_task": ms * 1e3 / st["tasks"],
-                              "span_us_per_task": st["span_ms"] * 1e3 / max(1, st["span_launches"]),
+                              "span_us_per_task": sum(st["k_span_ms"]) * 1e3 / max(1, sum(st["k_span_launches"])),
                               "sched_us_per_task": st["sched_ns"] / 1e3 / st["tasks"],
                               "launch_us_per_task": st["launch_ns"] / 1e3 / st["tasks"],
                               "retire_us_per_task": st["retire_ns"] / 1e3 / st["tasks"],
