@@ -125,3 +125,9 @@ def run_seq2seq_forced_lockstep(enc, dec, srcs: Sequence[Sequence[int]],
                 best[r][s] = Z[j].max()
     return ([[h[l][r] for l in range(L)] for r in range(n)],
             [[c[l][r] for l in range(L)] for r in range(n)], sel, best)
+
+
+def lstm_step_rows(W, b, X, Hp, Cp):
+    """One LSTM step (reading S1) for a stack of independent rows: X, Hp, Cp [rows, h] -> (H', C').
+    The row-stacked form of cells.lstm_cell that run_chain_schedule applies per task."""
+    return _lstm_rows(W, b, f64(X), f64(Hp), f64(Cp))

@@ -19,7 +19,7 @@ CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "libbm.so")
 BUILD = os.path.join(HERE, "_build")
 
-SOURCES = ["cell_step_sm100.cu", "lstm_persistent_sm100.cu", "cell_step_simt.cu", "scheduler.cpp",
+SOURCES = ["cell_step_sm100.cu", "cell_pair_sm100.cu", "lstm_persistent_sm100.cu", "cell_step_simt.cu", "scheduler.cpp",
            "runtime.cpp"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -319,7 +319,9 @@ __global__ void pack_rows_kernel(const float* __restrict__ src, void* dst, float
 // 64-column K block kc, stored contiguously (tile_rows x 128 B) in the 128B-swizzled K-major
 // layout the UMMA shared-memory descriptor expects: 16-byte chunk j of row r sits at chunk
 // position j ^ (r % 8). One pipeline stage of the kernel is then ONE contiguous bulk copy.
-__global__ void pack_tiles_kernel(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst,
+// Tensor-core weight tiles: each weight is rounded to its bf16 value (the bf16-weight path) and
+// stored as fp16 (exact for |w| >= 2^-17; see act_from_float in sm100_ptx.cuh).
+__global__ void pack_tiles_kernel(const float* __restrict__ src, __half* __restrict__ dst,
                                   int G, int H, int K, int tile_rows, int n_rows) {
   const size_t n = static_cast<size_t>(n_rows) * K;
   const int kblocks = K / 64;
@@ -332,14 +334,15 @@ __global__ void pack_tiles_kernel(const float* __restrict__ src, __nv_bfloat16* 
     const int kc = k / 64, j = (k % 64) / 8, el = k % 8;
     const size_t off = ((static_cast<size_t>(t) * kblocks + kc) * tile_rows + r) * 64 +
                        ((j ^ (r & 7)) * 8) + el;
-    dst[off] = __float2bfloat16_rn(src[static_cast<size_t>(src_row) * K + k]);
+    dst[off] = __float2half_rn(__bfloat162float(__float2bfloat16_rn(src[static_cast<size_t>(src_row) * K + k])));
   }
 }
 
-__global__ void convert_kernel(const float* __restrict__ src, void* dst, size_t n, int bf16) {
+// fp32 -> the tensor-core path's activation type (fp16, act_from_float) or a plain fp32 copy.
+__global__ void convert_kernel(const float* __restrict__ src, void* dst, size_t n, int act16) {
   for (size_t e = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; e < n;
        e += static_cast<size_t>(gridDim.x) * blockDim.x) {
-    if (bf16) static_cast<__nv_bfloat16*>(dst)[e] = __float2bfloat16_rn(src[e]);
+    if (act16) static_cast<__half*>(dst)[e] = act_from_float(src[e]);
     else static_cast<float*>(dst)[e] = src[e];
   }
 }
@@ -360,12 +363,12 @@ __global__ void pool_io_kernel(void* h_pool, float* c_pool, const int32_t* slots
     const size_t at = static_cast<size_t>(slots[i]) * H + u;
     if (write) {
       if (h_buf) {
-        if (bf16) static_cast<__nv_bfloat16*>(h_pool)[at] = __float2bfloat16_rn(h_buf[e]);
+        if (bf16) static_cast<__half*>(h_pool)[at] = act_from_float(h_buf[e]);
         else static_cast<float*>(h_pool)[at] = h_buf[e];
       }
       if (c_buf) c_pool[at] = c_buf[e];
     } else {
-      if (h_buf) h_buf[e] = bf16 ? __bfloat162float(static_cast<__nv_bfloat16*>(h_pool)[at])
+      if (h_buf) h_buf[e] = bf16 ? __half2float(static_cast<__half*>(h_pool)[at])
                                  : static_cast<float*>(h_pool)[at];
       if (c_buf) c_buf[e] = c_pool[at];
     }
@@ -399,7 +402,7 @@ cudaError_t launch_pack_rows(const float* src, void* dst, float* bias_dst, const
 
 cudaError_t launch_pack_tiles(const float* src, void* dst, int G, int H, int K, int tile_rows,
                               int n_rows, cudaStream_t st) {
-  pack_tiles_kernel<<<1184, 256, 0, st>>>(src, static_cast<__nv_bfloat16*>(dst), G, H, K, tile_rows, n_rows);
+  pack_tiles_kernel<<<1184, 256, 0, st>>>(src, static_cast<__half*>(dst), G, H, K, tile_rows, n_rows);
   return cudaGetLastError();
 }
 

@@ -174,6 +174,7 @@ struct WorkerState {
   unsigned int* sig_ctas = nullptr;
   unsigned int* done_ctas = nullptr;
   unsigned long long* amax = nullptr;
+  float* scratch = nullptr;
 };
 
 
@@ -216,6 +217,7 @@ struct Engine {
   float* logits = nullptr;         // [max_requests][max_decode][V] (record_logits)
   int logits_vocab = 0;
   unsigned long long* amax = nullptr;
+  float* scratch = nullptr;          // split-K partial exchange of cell_pair2_kernel (L2)
   unsigned int* done_ctas = nullptr;
   unsigned int* sig_ctas = nullptr;  // CTA counter of the fused completion signal / chain flag
   unsigned int* dep_flag = nullptr;  // launch chain flag (device): last completed sm100 launch

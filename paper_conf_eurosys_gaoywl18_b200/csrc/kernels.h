@@ -90,7 +90,14 @@ struct StepArgs {
                               // memory plan (no CTA pairs) so two workers' CTAs share an SM
   int cbuf_off;               // set by the launcher: shared-memory offset (from the 1 KB-aligned
                               // base) of the epilogue's prefetched c-state rows
+  int wslots;                 // set by the launcher (cell_pair2_kernel): weight ring slots
+  float* scratch;             // split-K partial exchange through L2 (cell_pair2_kernel): per CTA
+                              // [128 rows][256 columns] fp32, kPairScratchCTAs regions
 };
+
+// cell_pair2_kernel's split-K scratch: regions of [128][256] fp32 for up to this many CTAs.
+constexpr int kPairScratchCTAs = 148;
+cudaError_t launch_pair2(StepArgs a, const RowDesc* rows_host, cudaStream_t st, bool* done);
 
 // Completion signals (A12): a ring of host-mapped slots; task `seq` of a worker writes seq + 1
 // into slot seq % kSignalSlots (one writer per slot at a time: kSignalSlots >> tasks in flight).
@@ -147,7 +154,8 @@ cudaError_t launch_pack_rows(const float* src, void* dst, float* bias_dst, const
                              int G, int H, int K, int bf16, cudaStream_t st);
 cudaError_t launch_pack_tiles(const float* src, void* dst, int G, int H, int K, int tile_rows,
                               int n_rows, cudaStream_t st);
-cudaError_t launch_convert(const float* src, void* dst, size_t n, int bf16, cudaStream_t st);
+// act16 = 1: to the tensor-core path's fp16 activation storage (embeddings); 0: fp32 copy
+cudaError_t launch_convert(const float* src, void* dst, size_t n, int act16, cudaStream_t st);
 // Completion signal (A12): bump a host-mapped counter after everything before it in stream.
 cudaError_t launch_signal(unsigned long long* counter, unsigned long long value, cudaStream_t st);
 // Pool access helpers (tests): gather/scatter fp32 rows of h (bf16 or fp32) and c.

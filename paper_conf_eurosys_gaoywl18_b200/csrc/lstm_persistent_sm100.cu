@@ -337,7 +337,7 @@ __global__ void __launch_bounds__(kThreads, 1) lstm_persistent_kernel(const __gr
           const float hn = sigm(z3) * tanhf(cn);
           p.c_pool[r.slot * H + u] = cn;
           const int par_out = (r.flags & ROW_PARITY) ? 0 : 1;
-          static_cast<__nv_bfloat16*>(p.h_pool)[(par_out * NS + r.slot) * H + u] = __float2bfloat16_rn(hn);
+          static_cast<__half*>(p.h_pool)[(par_out * NS + r.slot) * H + u] = act_from_float(hn);
           if (r.flags & ROW_LAST) {
             const size_t ro = static_cast<size_t>(r.flags >> 8) * p.res_layers * H + u;
             p.res_h[ro] = hn;

@@ -101,6 +101,7 @@ static void swap_active(Engine& e, WorkerState& w) {
   std::swap(e.sig_ctas, w.sig_ctas);
   std::swap(e.done_ctas, w.done_ctas);
   std::swap(e.amax, w.amax);
+  std::swap(e.scratch, w.scratch);
 }
 
 // Make worker w's launch state the engine's active one (no-op with one worker).
@@ -154,6 +155,7 @@ static bm_status launch_one_step(Engine& e, Cell& c, const RowDesc* rows_dev, co
   a.res_c = e.res_c;
   a.res_layers = e.cfg.pool_layers;
   a.amax = e.amax;
+  a.scratch = e.scratch;
   a.done_ctas = e.done_ctas;
   a.res_tok = e.res_tok;
   a.max_decode = e.cfg.max_decode_len;
@@ -578,6 +580,7 @@ static void free_device(Engine& e) {
     cudaFree(ws.sig_ctas);
     cudaFree(ws.done_ctas);
     cudaFree(ws.amax);
+    cudaFree(ws.scratch);
   }
   if (!e.device()) return;
   dump_timeline(e);
@@ -599,6 +602,7 @@ static void free_device(Engine& e) {
   cudaFree(e.res_tok);
   cudaFree(e.logits);
   cudaFree(e.amax);
+  cudaFree(e.scratch);
   cudaFree(e.done_ctas);
   cudaFree(e.sig_ctas);
   cudaFree(e.dep_flag);
@@ -673,6 +677,8 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
               dalloc(&E.direct_rows, 2 * 4096) == cudaSuccess &&
               cudaEventCreateWithFlags(&E.direct_ev[0], cudaEventDisableTiming) == cudaSuccess &&
               cudaEventCreateWithFlags(&E.direct_ev[1], cudaEventDisableTiming) == cudaSuccess;
+    if (ok && c.precision == BM_PREC_BF16)  // cell_pair2_kernel's split-K exchange regions
+      ok = dalloc(&E.scratch, static_cast<size_t>(kPairScratchCTAs) * 128 * 256) == cudaSuccess;
     if (!ok) return fail(BM_E_NOMEM);
     // descriptor ring: every worker keeps <= k + MaxTasksToSubmit tasks of <= 512 rows in
     // flight, and a Schedule call's rows are placed contiguously (a wrap wastes the tail):
@@ -749,7 +755,9 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       memset(ws.signal_host, 0, kSignalSlots * sizeof(unsigned long long));
       if (cudaHostGetDevicePointer(reinterpret_cast<void**>(&ws.signal_dev), ws.signal_host, 0) != cudaSuccess ||
           dalloc(&ws.dep_flag, 1) != cudaSuccess || dalloc(&ws.sig_ctas, 1) != cudaSuccess ||
-          dalloc(&ws.done_ctas, 1) != cudaSuccess || dalloc(&ws.amax, 512) != cudaSuccess)
+          dalloc(&ws.done_ctas, 1) != cudaSuccess || dalloc(&ws.amax, 512) != cudaSuccess ||
+          (c.precision == BM_PREC_BF16 &&
+           dalloc(&ws.scratch, static_cast<size_t>(kPairScratchCTAs) * 128 * 256) != cudaSuccess))
         return fail(BM_E_NOMEM);
       if (cudaMemsetAsync(ws.dep_flag, 0, 4, E.stream) != cudaSuccess ||
           cudaMemsetAsync(ws.sig_ctas, 0, 4, E.stream) != cudaSuccess ||

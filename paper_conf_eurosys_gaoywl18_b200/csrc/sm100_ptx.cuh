@@ -2,11 +2,23 @@
 // cp.async, tcgen05 MMA / TMEM, clusters, PDL). Device code only.
 #pragma once
 #include <cuda_bf16.h>
+#include <cuda_fp16.h>
 #include <stdint.h>
 
 #include "kernels.h"
 
 namespace bm {
+// Operands of the tensor-core path (BM_PREC_BF16): fp16 storage. Activations (pool h, the
+// embedding rows) are fp16: h = o * tanh(c) lies in (-1, 1) and the embeddings are O(1), so
+// fp16's 10-bit mantissa (8x finer than bf16's 7 bits) costs nothing in range; the recurrence
+// feeds each step's rounded h into the next step, and over the longest configs[2] requests
+// (~200 + 200 steps, 4 layers) bf16 activations drift up to 0.034 from the exact result while
+// fp16 ones stay at 0.002 (precision reading), against north_star's 5e-3. The
+// weights keep bf16 VALUES (generated bf16-representable and fp16-exact, workloads/gen.py;
+// user weights are rounded to bf16 first) and are stored as fp16 -- exactly -- because the
+// MMA takes one type for A and B.
+__device__ __forceinline__ __half act_from_float(float x) { return __float2half_rn(x); }
+
 namespace ptx {
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -148,9 +160,10 @@ __device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
   d |= static_cast<uint64_t>(2) << 61;            // SWIZZLE_128B
   return d;
 }
-// Instruction descriptor, kind::f16: D fp32, A bf16, B bf16, both K-major, M x N.
+// Instruction descriptor, kind::f16: D fp32, A and B fp16 (kind::f16 takes one operand type for
+// both: a bf16 x fp16 descriptor is an illegal instruction on sm_100a), both K-major, M x N.
 __device__ __forceinline__ uint32_t idesc_bf16(int M, int N) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(N >> 3) << 17) |
+  return (1u << 4) | (0u << 7) | (0u << 10) | (static_cast<uint32_t>(N >> 3) << 17) |
          (static_cast<uint32_t>(M >> 4) << 24);
 }
 __device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc,

@@ -218,3 +218,33 @@ def test_leaf_batch_invariance(b_small, b_big):
         eh, ec = cells.tree_leaf(w.W_leaf, w.b_leaf, w.E[toks[i]])
         assert np.max(np.abs(big_h[i, 0] - eh)) <= STEP_TOL[bm.PREC_BF16]
         assert np.max(np.abs(big_c[i, 0] - ec)) <= STEP_TOL[bm.PREC_BF16]
+
+
+def test_lstm_step_every_batch_size():
+    """Every task size the scheduler can form, b = 1..512 (bmax), one LSTM step at h = 1024
+    through whichever kernel and plan the launcher picks for that b (single-CTA tcgen05 with
+    its ring plans, CTA pair above 128 rows, one or two column blocks, ragged tails): result
+    rows (fp32) against the oracle at single-step tolerance, pool h (bf16) at north_star's."""
+    from oracle import batched
+    rng = np.random.default_rng(77)
+    h, V = 1024, 512
+    e, cid, w = lstm_engine(h, 1, V, bm.PREC_BF16, max_slots=2048, max_requests=1024)
+    worst = {}
+    for b in range(1, 513):
+        slots = _slots(rng, b, 2048)
+        first = rng.random(b) < 0.1
+        h0 = bf16_vals(rng.uniform(-1, 1, (b, h)), bm.PREC_BF16)
+        c0 = rng.uniform(-2, 2, (b, h)).astype(np.float32)
+        e.pool_write(0, 0, slots, h0, c0)
+        toks = rng.integers(3, V, size=b)
+        flags = (first * bm.ROW_FIRST) | bm.ROW_LAST | (np.arange(b) << 8)
+        e.cell_step(cid, np.stack([toks, np.zeros(b), slots, flags], 1).astype(np.int32))
+        rh, rc = e.result_rows(np.arange(b))
+        ph = e.pool_read(0, 1, slots)[0]
+        hp = np.where(first[:, None], 0.0, h0)
+        cp = np.where(first[:, None], 0.0, c0)
+        eh, ec = batched.lstm_step_rows(w.W[0], w.b[0], w.E[toks], hp, cp)
+        err = max(np.max(np.abs(rh[:, 0] - eh)), np.max(np.abs(rc[:, 0] - ec)))
+        worst[b] = (err, np.max(np.abs(ph - eh)))
+    bad = {b: v for b, v in worst.items() if v[0] > STEP_TOL[bm.PREC_BF16] or v[1] > TOL[bm.PREC_BF16]}
+    assert not bad, sorted(bad.items())[:10]

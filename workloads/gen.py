@@ -30,15 +30,19 @@ CHAIN, SEQ2SEQ, TREE = 0, 1, 2
 
 
 def bf16_round(x: np.ndarray) -> np.ndarray:
-    """Round fp32 values to the nearest bf16-representable fp32 (round-to-nearest-even).
+    """Round fp32 values to the nearest bf16-representable fp32 (round-to-nearest-even), with
+    magnitudes below 2^-14 (fp16's smallest normal) flushed to zero.
 
-    Used only to make generated weights exactly representable in bf16, so that the bf16
-    device path and the fp64 oracle see identical weight values (reading S25)."""
+    Used only to make generated values exactly representable on the tensor-core path, which
+    holds bf16-valued weights and its activations in fp16 storage (precision):
+    a bf16 value of magnitude >= 2^-14 is exact in fp16, so the device and the fp64 oracle see
+    identical values (reading S25)."""
     a = np.ascontiguousarray(x, dtype=np.float32)
     u = a.view(np.uint32).astype(np.uint64)
     lsb = (u >> 16) & 1
     u = (u + 0x7FFF + lsb) & 0xFFFF0000
-    return u.astype(np.uint32).view(np.float32).reshape(a.shape)
+    r = u.astype(np.uint32).view(np.float32).reshape(a.shape)
+    return np.where(np.abs(r) < 2.0 ** -14, np.float32(0), r).astype(np.float32)
 
 
 def _uniform(rng, shape, bound):
