@@ -58,7 +58,8 @@ constexpr int kMaxS = 4;                // max split-K cluster size (K = 2h = 20
 //  * activations: one 64-wide K block per stage, gathered by 256 threads with cp.async (the
 //    LSU path runs beside the TMA engine).
 constexpr int kWChunkMax = 4;           // K blocks per weight chunk, large tasks (64 KB chunks)
-constexpr int kWRing = 2;               // weight chunks in the ring
+constexpr int kWRing = 2;               // weight chunks in the CTA-pair kernel's ring
+constexpr int kWRingMax = 4;            // single-CTA kernel: up to 4 slots (StepArgs::wslots)
 // Small tasks (npad <= 128) use 32 KB weight chunks and a 32 KB activation ring so the CTA fits
 // in ~100 KB and two CTAs share an SM: under PDL the next launch's weight stream and gather
 // overlap this launch's split-K epilogue. Larger tasks use 64 KB chunks and a 64 KB ring.
@@ -73,8 +74,9 @@ __host__ __device__ __forceinline__ int x_stages_for(int npad, int xring) {
 // wblk = one K block of the CTA's weight tile (tile rows x 128 B: 16 KB LSTM / projection,
 // 12 KB leaf, 10 KB internal)
 // xkb = K blocks per activation stage (one hand-off per stage)
-__host__ __device__ __forceinline__ int region_bytes(int pcols, int wcb, int xring, int wblk, int xkb, int npad) {
-  const int a = kWRing * wcb * wblk + x_stages_for(npad * xkb, xring) * npad * xkb * 128;
+__host__ __device__ __forceinline__ int region_bytes(int pcols, int wcb, int xring, int wblk, int xkb, int npad,
+                                                     int wslots) {
+  const int a = wslots * wcb * wblk + x_stages_for(npad * xkb, xring) * npad * xkb * 128;
   const int b = 129 * pcols * 4 + 4 * 128 * 4;  // partial / logits tile of pcols columns
   return a > b ? a : b;
 }
@@ -120,14 +122,18 @@ __global__ void __launch_bounds__(kThreads, 2)
   const uint32_t full0 = smem_u32(bars);                            // activation stage full
   const uint32_t empty0 = smem_u32(bars + kMaxStages);              // activation stage free
   const uint32_t wfull0 = smem_u32(bars + 2 * kMaxStages);          // weight chunk landed
-  const uint32_t wempty0 = smem_u32(bars + 2 * kMaxStages + kWRing);  // weight chunk free
-  const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages + 2 * kWRing);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 2 * kWRing + 1);
+  const uint32_t wempty0 = smem_u32(bars + 2 * kMaxStages + kWRingMax);  // weight chunk free
+  const uint32_t done_bar = smem_u32(bars + 2 * kMaxStages + 2 * kWRingMax);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kMaxStages + 2 * kWRingMax + 1);
+  // weight ring slots: slot w is filled by lane w of the TMA warp -- one thread's bulk copies
+  // complete one after another (~0.6 us each), copies of different threads overlap
+  // (tools/stream_bench.cu mode 8)
+  const int wr = p.wslots > 0 ? p.wslots : kWRing;
   int* flag_last = reinterpret_cast<int*>(tmem_slot + 1);
   RowDesc* rtab = reinterpret_cast<RowDesc*>(base + 1024);  // this CTA's rows (col0 + c)
   uint8_t* smem = base + kTailBytes;                      // 1024-aligned (kTailBytes = 5 KB)
-  uint8_t* w_ring = smem;                                 // kWRing x wcb x 16 KB
-  uint8_t* x_st = smem + (wcpa ? 0 : kWRing * wcb * wblk_bytes);  // kStages x stage
+  uint8_t* w_ring = smem;                                 // wr x wcb x wblk
+  uint8_t* x_st = smem + (wcpa ? 0 : wr * wcb * wblk_bytes);  // kStages x stage
   const int x_blk_bytes = npad * 128;                     // one K block of the activation tile
   const int x_stage_bytes = x_blk_bytes * xkb + (wcpa ? wblk_bytes * xkb : 0);
 
@@ -140,8 +146,8 @@ __global__ void __launch_bounds__(kThreads, 2)
       mbar_init(full0 + 8 * s, kProducerThreads);  // every gather thread's cp.async arrive
       mbar_init(empty0 + 8 * s, 1);
     }
-    for (int s = 0; s < kWRing; ++s) {
-      mbar_init(wfull0 + 8 * s, 1);   // the TMA thread's arrive.expect_tx
+    for (int s = 0; s < kWRingMax; ++s) {
+      mbar_init(wfull0 + 8 * s, 1);   // the TMA lane's arrive.expect_tx
       mbar_init(wempty0 + 8 * s, 1);
     }
     mbar_init(done_bar, 1);
@@ -254,13 +260,13 @@ __global__ void __launch_bounds__(kThreads, 2)
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
     // Weights are read-only: streaming starts before griddepcontrol.wait (PDL overlap).
-    if (!wcpa && lane == 0) {
+    if (!wcpa && lane < wr) {
       const int kblocks = (p.K0 + p.K1) / kBK;
       const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
                             (static_cast<size_t>(blockIdx.y) * kblocks + k_begin / kBK) * wblk_bytes;
-      for (int c = 0; c < n_chunks; ++c) {
-        const int s = c % kWRing;
-        const int round = c / kWRing;
+      for (int c = lane; c < n_chunks; c += wr) {
+        const int s = c % wr;
+        const int round = c / wr;
         if (round > 0) mbar_wait(wempty0 + 8 * s, (round - 1) & 1);
         const int nblk = min(kpc, nk - c * kpc);
         const uint32_t bytes = static_cast<uint32_t>(nblk * wblk_bytes);
@@ -292,9 +298,9 @@ __global__ void __launch_bounds__(kThreads, 2)
       for (int j = 0; j < xkb; ++j) {
         const int kb = st * xkb + j;
         const int c = kb / kpc;
-        const int ws = c % kWRing;
+        const int ws = c % wr;
         if (!wcpa && kb % kpc == 0) {
-          mbar_wait_warp(wfull0 + 8 * ws, (c / kWRing) & 1);
+          mbar_wait_warp(wfull0 + 8 * ws, (c / wr) & 1);
           tc_fence_after();
           if (lane == 0 && c < 4) phase_mark(p, 28 + c);  // weight chunk c at the MMA
           if (lane == 0 && kb == 0) phase_mark(p, 13);
@@ -670,6 +676,22 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
     a.wcpa = 1;
     a.xkb = 1;
   }
+  // weight ring slots, one TMA lane each (bulk copies of one thread complete one at a time)
+  a.wslots = kWRing;
+  static const int env_wslots = getenv("BM_WSLOTS") ? atoi(getenv("BM_WSLOTS")) : 0;
+  // projection up to 64 rows (BM_PROJ_TMA, default on): the 256 KB vocab tile through a
+  // 4 x 16 KB TMA ring filled by four lanes (instead of the producers' cp.async, which fills
+  // one stage at a time), two CTAs per SM (<= 113 KB); -1 us per launch at b <= 64, +1.7 us at
+  // 128 (profiles/round2/kbench_wslots_r2o.log), so larger tasks keep the cp.async plan
+  static const int env_proj_tma = getenv("BM_PROJ_TMA") ? atoi(getenv("BM_PROJ_TMA")) : 1;
+  if (proj_small && env_proj_tma && npad <= 64) {
+    a.wcpa = 0;
+    a.wcb = 1;
+    a.wslots = 4;
+    a.xkb = npad <= 64 ? 2 : 1;
+    a.xring = 2 * a.xkb * npad * 128;
+  }
+  if (env_wslots >= 1 && env_wslots <= kWRingMax) a.wslots = env_wslots;
   const int nk_all = a.kslice / kBK;
   if (EPI == EPI_PROJ) {
     if (a.xkb > 1 && (a.H / kBK) % a.xkb != 0) a.xkb = 1;
@@ -699,7 +721,8 @@ cudaError_t launch_impl(StepArgs a, const RowDesc* rows_host, cudaStream_t st) {
     }
   }
   if (!a.wcpa)
-    a.cbuf_off = kTailBytes + region_bytes(a.pchunk > 0 ? a.pchunk : npad, a.wcb, a.xring, wblk, a.xkb, npad);
+    a.cbuf_off = kTailBytes + region_bytes(a.pchunk > 0 ? a.pchunk : npad, a.wcb, a.xring, wblk, a.xkb, npad,
+                                           a.wslots);
   const size_t smem = 1024 + a.cbuf_off + cbuf_bytes;
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   const int tiles = EPI == EPI_PROJ ? a.W_rows / 128 : a.H / a.U;

@@ -90,7 +90,7 @@ struct StepArgs {
                               // memory plan (no CTA pairs) so two workers' CTAs share an SM
   int cbuf_off;               // set by the launcher: shared-memory offset (from the 1 KB-aligned
                               // base) of the epilogue's prefetched c-state rows
-  int wslots;                 // set by the launcher (cell_pair2_kernel): weight ring slots
+  int wslots;                 // set by the launcher: weight ring slots (one TMA lane each)
   float* scratch;             // split-K partial exchange through L2 (cell_pair2_kernel): per CTA
                               // [128 rows][256 columns] fp32, kPairScratchCTAs regions
 };
