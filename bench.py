@@ -496,16 +496,23 @@ def run_workload(ctx, a, wl, n_req, steps, warmup, headline):
         unit = make_trace(wl, sweep_n, 1.0, seed=ctx.shard.rank_seed(100, rank))   # unit-rate Poisson
         pu = e.prepare_requests(unit, cells)
         fracs = WL[wl]["fracs"] if not a.quick else (0.05, 0.5, 0.8, 0.95)
-        for f in fracs:
-            lam = f * mu
+        def point(lam):
             n_pt = int(min(sweep_n, max(2000, math.ceil(POINT_SECONDS * lam))))
             pp = pu if n_pt == sweep_n else e.prepare_requests(unit[:n_pt], cells)
-            curve.append(measure_point(ctx, e, pp, n_pt, lam))
+            return measure_point(ctx, e, pp, n_pt, lam)
+        for f in fracs:
+            curve.append(point(f * mu))
         bound_ms = (a.p90_ms if headline else 0) or WL[wl]["p90_ms"]
         knee_ms = 2.0 * curve[0]["p90_ms"]
         if not bound_ms:
             bound_ms = knee_ms
             bound_kind = "knee (2x lowest-load p90)"
+        # the burst estimate mu can sit below the sustainable rate: extend the grid upwards
+        # until a point fails (not sustained, or p90 above the bound)
+        extra = 0
+        while (not a.quick and extra < 6 and curve[-1]["sustained"] and curve[-1]["p90_ms"] <= bound_ms):
+            curve.append(point(curve[-1]["offered"] * 1.1))
+            extra += 1
 
         def ok(c, b):
             return c["sustained"] and c["p90_ms"] <= b
@@ -519,9 +526,7 @@ def run_workload(ctx, a, wl, n_req, steps, warmup, headline):
         hi = min(above) if above else None
         for _ in range(2 if (hi is not None and not a.quick) else 0):
             mid = 0.5 * (lo + hi)
-            n_pt = int(min(sweep_n, max(2000, math.ceil(POINT_SECONDS * mid))))
-            pp = pu if n_pt == sweep_n else e.prepare_requests(unit[:n_pt], cells)
-            c = measure_point(ctx, e, pp, n_pt, mid)
+            c = point(mid)
             c["bisection"] = True
             curve.append(c)
             lo, hi = (mid, hi) if ok(c, bound_ms) else (lo, mid)

@@ -98,6 +98,16 @@ typedef struct {
                              /* request sharding's one worker per GPU (default). >1 needs */
                              /* policy CELLULAR and persistent 0; the bf16 LSTM launches  */
                              /* then use a <= 113 KB plan so two workers' CTAs share SMs. */
+  int devices;               /* device contexts the workers spread over (§8f N2, the paper's */
+                             /* multi-GPU design, L317, L337): worker w runs on context w %  */
+                             /* devices, context c on CUDA device (device + c) % count. A    */
+                             /* context holds its own weight replica and state pool; when a  */
+                             /* subgraph is scheduled on a worker of another context (it is  */
+                             /* unpinned: nothing of it in flight, L381), its state rows move */
+                             /* with it by peer copies ("if the execution of successive cells */
+                             /* switch from one GPU to another, one must copy data", L337),  */
+                             /* counted in bm_stats.migrations. Results land on context 0.  */
+                             /* 1 = one context (default); > 1 needs workers >= devices.    */
   double roof_hbm_gbs;       /* time_kernels: the roofline denominators (bench.py passes     */
   double roof_tc_tflops;     /* MEASURED_PEAKS.json); 0 = bm_stats.k_roof_* stay 0          */
 } bm_config;
@@ -110,7 +120,8 @@ enum {
 
 /* Fill *cfg with defaults: device 0, BF16, WALL, hidden 1024, 1 layer, 65536 slots,
  * 65536 requests, MaxTasksToSubmit 5, Min 1, k 0, max_decode_len 512, keep_results 0,
- * record_log 1, persistent 0, policy BM_POLICY_CELLULAR, bucket_width 10, workers 1. */
+ * record_log 1, persistent 0, policy BM_POLICY_CELLULAR, bucket_width 10, workers 1,
+ * devices 1. */
 void bm_config_default(bm_config* cfg);
 
 /* ---------------------------------------------------------------- cells (bm_load_cell) */
@@ -332,6 +343,8 @@ typedef struct {
   double k_roof_hbm_ms[BM_K_CLASSES];     /* sum of bytes / roof_hbm_gbs                 */
   double k_roof_tc_ms[BM_K_CLASSES];      /* sum of flops / roof_tc_tflops               */
   double k_roof_ms[BM_K_CLASSES];         /* sum of max(the two) per launch              */
+  uint64_t migrations;       /* state rows moved between device contexts (bm_config.devices) */
+  double migration_bytes;    /* bytes those peer copies moved                               */
 } bm_stats;
 
 bm_status bm_get_stats(bm_engine* e, bm_stats* out);

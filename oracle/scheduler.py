@@ -124,12 +124,22 @@ class Task:
     finish: float = 0.0
 
 
+def _input_slots(r: "Req", node: int) -> List[int]:
+    """State slots a node reads: a chain / Seq2Seq node after the request's first reads the
+    request's own (h, c); a tree internal node reads its two children's; a leaf reads none."""
+    if r.kind == TREE:
+        if r.left[node] < 0:
+            return []
+        return [r.slots[r.left[node]], r.slots[r.right[node]]]
+    return [] if node == 0 else [r.slots[-1]]
+
+
 class Replay:
     """Algorithm 1 with one worker per engine (S23), driven by `run()` in virtual time."""
 
     def __init__(self, cell_types: Sequence[Tuple[int, int]], max_slots: int = 1 << 20,
                  max_tasks_to_submit: int = 5, min_followon: int = 1,
-                 schedule_when_outstanding_leq: int = 0, workers: int = 1):
+                 schedule_when_outstanding_leq: int = 0, workers: int = 1, devices: int = 1):
         # cell_types: list of (bmax, priority); cell id = position
         self.cts = [CellType(i, bm, pr) for i, (bm, pr) in enumerate(cell_types)]
         self.pool = SlotPool(max_slots)
@@ -145,6 +155,22 @@ class Replay:
         self.completions: List[Tuple[int, float]] = []   # (rid, tick) in completion order
         self.now = 0.0
         self.last_finish_w = [0.0] * workers
+        # §8f N2 across GPUs: worker w runs on device w % devices; a task row whose input state
+        # was last written on another device needs that state copied over first ("if the
+        # execution of successive cells switch from one GPU to another, one must copy data from
+        # one GPU to another", L337). Counted per input slot moved.
+        self.devices = devices
+        self.slot_dev: Dict[int, int] = {}
+        self.migrations = 0
+
+    def _count_migrations(self, task: "Task", dev: int):
+        """§8f N2: input state rows of the task last written on another device (L337)."""
+        for row in task.rows:
+            for s in _input_slots(self.reqs[row.rid], row.node):
+                if self.slot_dev.get(s, dev) != dev:
+                    self.migrations += 1
+        for row in task.rows:
+            self.slot_dev[row.slot] = dev
 
     # ------------------------------------------------------------ request processor (A1)
     def admit(self, kind: int, cells: Sequence[int], length: int = 0, decode_len: int = 0,
@@ -403,6 +429,7 @@ class Replay:
             for w in range(self.W):   # Schedule(worker) for every idle worker, in id order
                 if len(self.inflight_w[w]) <= self.k:
                     for task in self.schedule(w):
+                        self._count_migrations(task, w % self.devices)
                         start = max(t, self.last_finish_w[w])
                         task.finish = start + 1
                         self.last_finish_w[w] = task.finish

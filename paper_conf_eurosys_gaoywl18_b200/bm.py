@@ -36,7 +36,7 @@ class Config(C.Structure):
         "device", "precision", "clock", "hidden", "pool_layers", "max_slots", "max_requests",
         "max_tasks_to_submit", "min_followon_batch", "schedule_when_outstanding_leq",
         "max_decode_len", "keep_results", "record_logits", "time_kernels", "record_log",
-        "persistent", "policy", "bucket_width", "workers")] + [
+        "persistent", "policy", "bucket_width", "workers", "devices")] + [
         ("roof_hbm_gbs", C.c_double), ("roof_tc_tflops", C.c_double)]
 
 
@@ -94,7 +94,8 @@ class Stats(C.Structure):
                 ("launch_ns", C.c_double), ("retire_ns", C.c_double),
                 ("k_launches", C.c_uint64 * K_CLASSES), ("k_span_launches", C.c_uint64 * K_CLASSES)] + [
         (n, C.c_double * K_CLASSES) for n in ("k_span_ms", "k_rows", "k_bytes", "k_flops", "k_roof_hbm_ms",
-                                              "k_roof_tc_ms", "k_roof_ms")]
+                                              "k_roof_tc_ms", "k_roof_ms")] + [
+        ("migrations", C.c_uint64), ("migration_bytes", C.c_double)]
 
 
 class LaunchRecord(C.Structure):

@@ -138,6 +138,34 @@ struct Cell {
   int running_tasks = 0;     // NumRunningTasks (S17)
 };
 
+// Device context (bm_config.devices, §8f N2): the state pool, descriptor ring and the weight
+// replica of every cell on one CUDA device. The Engine's own fields (h_pool, c_pool, tok, dead,
+// ring_dev, ..., Cell::W/bias/E/W_out/b_out) are the ACTIVE context's; select_worker() swaps
+// them with the parked copies here when the next worker lives on another context.
+struct CellWeights {
+  std::vector<void*> W;
+  std::vector<float*> bias;
+  void* E = nullptr;
+  void* W_out = nullptr;
+  float* b_out = nullptr;
+};
+struct DevCtx {
+  int cuda_dev = 0;
+  void* h_pool = nullptr;
+  float* c_pool = nullptr;
+  int* tok = nullptr;
+  int* dead = nullptr;
+  RowDesc* ring_dev = nullptr;
+  RowDesc* ring_host = nullptr;
+  int ring_head = 0;
+  unsigned int* rows_flag_dev = nullptr;
+  unsigned int* rows_seq_host = nullptr;
+  unsigned int rows_seq = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t copy_ev = nullptr;
+  std::vector<CellWeights> cells;
+};
+
 struct TaskRow {
   int req;     // request table index
   int node;
@@ -273,6 +301,12 @@ struct Engine {
   // workers (§8f N2): parked launch state of the inactive workers; `cur` is active
   std::vector<WorkerState> parked;
   int cur = 0;
+  // device contexts (bm_config.devices): parked state of the inactive contexts, the context
+  // of each worker, and the context holding each slot's latest state (-1: none yet)
+  std::vector<DevCtx> ctxs;
+  int cur_ctx = 0;
+  std::vector<int> worker_ctx;
+  std::vector<int8_t> slot_ctx;
   uint64_t tasks_total = 0;         // tasks over all workers (task log index)
 
   bool device() const { return cfg.clock != BM_CLOCK_DRY; }

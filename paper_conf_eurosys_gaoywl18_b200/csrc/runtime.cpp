@@ -104,12 +104,97 @@ static void swap_active(Engine& e, WorkerState& w) {
   std::swap(e.scratch, w.scratch);
 }
 
-// Make worker w's launch state the engine's active one (no-op with one worker).
+// Device contexts (§8f N2): swap the active context's pool / ring / weights with a parked one.
+static void swap_ctx(Engine& e, DevCtx& c) {
+  std::swap(e.h_pool, c.h_pool);
+  std::swap(e.c_pool, c.c_pool);
+  std::swap(e.tok, c.tok);
+  std::swap(e.dead, c.dead);
+  std::swap(e.ring_dev, c.ring_dev);
+  std::swap(e.ring_host, c.ring_host);
+  std::swap(e.ring_head, c.ring_head);
+  std::swap(e.rows_flag_dev, c.rows_flag_dev);
+  std::swap(e.rows_seq_host, c.rows_seq_host);
+  std::swap(e.rows_seq, c.rows_seq);
+  std::swap(e.copy_stream, c.copy_stream);
+  std::swap(e.copy_ev, c.copy_ev);
+  c.cells.resize(e.cells.size());
+  for (size_t i = 0; i < e.cells.size(); ++i) {
+    Cell& a = e.cells[i];
+    CellWeights& b = c.cells[i];
+    std::swap(a.W, b.W);
+    std::swap(a.bias, b.bias);
+    std::swap(a.E, b.E);
+    std::swap(a.W_out, b.W_out);
+    std::swap(a.b_out, b.b_out);
+  }
+}
+
+static void select_ctx(Engine& e, int c) {
+  if (c == e.cur_ctx || e.ctxs.size() < 2) return;
+  swap_ctx(e, e.ctxs[e.cur_ctx]);
+  swap_ctx(e, e.ctxs[c]);
+  e.cur_ctx = c;
+  if (e.device()) cudaSetDevice(e.ctxs[c].cuda_dev);
+}
+
+// Make worker w's launch state (and its device context) the engine's active one (no-op with
+// one worker).
 void select_worker(Engine& e, int w) {
   if (w == e.cur || e.parked.empty()) return;
   swap_active(e, e.parked[e.cur]);
   swap_active(e, e.parked[w]);
   e.cur = w;
+  select_ctx(e, e.worker_ctx.empty() ? 0 : e.worker_ctx[w]);
+}
+
+// §8f N2 state migration (L337): before a task runs on the active context, every input state
+// row it reads that another context wrote last (its subgraph moved: unpinned, nothing in
+// flight, L381) is copied over -- h of both parities and c of every pool layer, the feed token
+// and the <eos> mark -- on the active worker's stream, ahead of the task's kernels. The producer
+// of that state has retired (pinning), so its writes are complete.
+static bm_status migrate_inputs(Engine& e, std::vector<Task>& tasks) {
+  if (e.ctxs.size() < 2) return BM_OK;
+  const int to = e.cur_ctx;
+  const size_t H = e.H(), S = e.cfg.max_slots, L = e.cfg.pool_layers, el = e.elem();
+  auto move = [&](int slot) -> bm_status {
+    const int from = e.slot_ctx[slot];
+    if (from < 0 || from == to) return BM_OK;
+    e.stats.migrations += 1;
+    e.stats.migration_bytes += static_cast<double>(L * (2 * H * el + H * 4) + 8);
+    if (e.device()) {
+      const DevCtx& src = e.ctxs[from];
+      const int dd = e.ctxs[to].cuda_dev, sd = src.cuda_dev;
+      for (size_t l = 0; l < L; ++l) {
+        for (size_t par = 0; par < 2; ++par) {
+          const size_t off = ((l * 2 + par) * S + slot) * H * el;
+          CK(cudaMemcpyPeerAsync(static_cast<char*>(e.h_pool) + off, dd, static_cast<const char*>(src.h_pool) + off,
+                                 sd, H * el, e.stream));
+        }
+        const size_t coff = (l * S + slot) * H;
+        CK(cudaMemcpyPeerAsync(e.c_pool + coff, dd, src.c_pool + coff, sd, H * 4, e.stream));
+      }
+      CK(cudaMemcpyPeerAsync(e.tok + slot, dd, src.tok + slot, sd, 4, e.stream));
+      CK(cudaMemcpyPeerAsync(e.dead + slot, dd, src.dead + slot, sd, 4, e.stream));
+      e.pdl_ok = false;  // copies precede the next launch on this stream: full ordering
+    }
+    return BM_OK;
+  };
+  for (Task& t : tasks) {
+    const int epi = e.cells[t.ct].epi;
+    for (const RowDesc& r : t.desc) {
+      bm_status st = BM_OK;
+      if (epi == EPI_INTERNAL) {          // children's h / c by slot
+        st = move(r.a);
+        if (st == BM_OK) st = move(r.b);
+      } else if (epi == EPI_LSTM && !(r.flags & ROW_FIRST)) {  // the request's own state
+        st = move(r.slot);
+      }
+      if (st != BM_OK) return st;
+    }
+    for (const RowDesc& r : t.desc) e.slot_ctx[r.slot] = static_cast<int8_t>(to);
+  }
+  return BM_OK;
 }
 
 // ---------------------------------------------------------------- launching tasks
@@ -475,7 +560,8 @@ static bm_status schedule_and_launch_one(Engine& e, int* n_tasks) {
   e.stats.schedule_calls += 1;
   if (tasks.empty()) return BM_OK;
   const auto t1 = std::chrono::steady_clock::now();
-  bm_status s = launch_tasks(e, tasks);
+  bm_status s = migrate_inputs(e, tasks);
+  if (s == BM_OK) s = launch_tasks(e, tasks);
   e.stats.launch_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t1).count();
   if (s != BM_OK) return s;
   for (Task& t : tasks) e.inflight.push_back(std::move(t));
@@ -549,6 +635,7 @@ void bm_config_default(bm_config* c) {
   c->policy = BM_POLICY_CELLULAR;
   c->bucket_width = 10;
   c->workers = 1;
+  c->devices = 1;
 }
 
 static void dump_timeline(Engine& e) {
@@ -569,6 +656,29 @@ static void dump_timeline(Engine& e) {
 
 static void free_device(Engine& e) {
   select_worker(e, 0);
+  for (size_t ci = 1; ci < e.ctxs.size(); ++ci) {
+    DevCtx& x = e.ctxs[ci];
+    if (!e.device()) break;
+    cudaSetDevice(x.cuda_dev);
+    cudaFree(x.h_pool);
+    cudaFree(x.c_pool);
+    cudaFree(x.tok);
+    cudaFree(x.dead);
+    cudaFree(x.ring_dev);
+    cudaFree(x.rows_flag_dev);
+    if (x.ring_host) cudaFreeHost(x.ring_host);
+    if (x.rows_seq_host) cudaFreeHost(x.rows_seq_host);
+    if (x.copy_stream) cudaStreamDestroy(x.copy_stream);
+    if (x.copy_ev) cudaEventDestroy(x.copy_ev);
+    for (CellWeights& w : x.cells) {
+      for (void* p : w.W) cudaFree(p);
+      for (float* p : w.bias) cudaFree(p);
+      cudaFree(w.E);
+      cudaFree(w.W_out);
+      cudaFree(w.b_out);
+    }
+  }
+  if (e.device() && e.ctxs.size() > 1) cudaSetDevice(e.ctxs[0].cuda_dev);
   for (size_t w = 1; w < e.parked.size(); ++w) {
     WorkerState& ws = e.parked[w];
     if (ws.stream) {
@@ -635,6 +745,7 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       c.max_tasks_to_submit < 1 || c.min_followon_batch < 1 || c.schedule_when_outstanding_leq < 0 ||
       c.max_decode_len < 1 || c.precision < 0 || c.precision > 1 || c.clock < 0 || c.clock > 2 ||
       c.policy < 0 || c.policy > 1 || c.bucket_width < 1 || c.workers < 1 || c.workers > 8 ||
+      c.devices < 1 || c.devices > c.workers || (c.devices > 1 && c.persistent) ||
       (c.workers > 1 && c.policy != BM_POLICY_CELLULAR) ||
       // tasks in flight per worker (<= k + MaxTasksToSubmit) must fit the completion-signal
       // ring and the persistent kernel's task-header ring (both kSignalSlots = 256 entries)
@@ -648,6 +759,11 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
   for (int i = 0; i < c.max_slots; ++i) e->free_slots_heap[i] = i;  // sorted == valid min-heap
   e->t0 = std::chrono::steady_clock::now();
   if (c.workers > 1) e->parked.resize(c.workers);
+  // device contexts (§8f N2): worker w on context w % devices; every slot starts nowhere
+  e->ctxs.resize(c.devices);
+  e->worker_ctx.resize(c.workers);
+  for (int w = 0; w < c.workers; ++w) e->worker_ctx[w] = w % c.devices;
+  e->slot_ctx.assign(c.max_slots, -1);
   if (e->device()) {
     Engine& E = *e;
     auto fail = [&](bm_status s) {
@@ -745,9 +861,45 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
       E.tl_retire.assign(Engine::kTimeline, 0);
       E.tl_b.assign(Engine::kTimeline, 0);
     }
-    // workers 1..W-1 (§8f N2): own stream, completion counter, launch chain, device scratch
+    // device contexts 1..D-1 (§8f N2): CUDA device (device + c) % count, each with its own
+    // state pool, descriptor ring and copy stream (the weight replicas follow in bm_load_cell);
+    // peer access lets every context's kernels write the result rows on context 0
+    for (int ci = 0; ci < c.devices; ++ci) E.ctxs[ci].cuda_dev = (c.device + ci) % ndev;
+    for (int ci = 1; ci < c.devices; ++ci) {
+      DevCtx& x = E.ctxs[ci];
+      if (cudaSetDevice(x.cuda_dev) != cudaSuccess) return fail(BM_E_CUDA);
+      if (x.cuda_dev != c.device) {
+        cudaDeviceEnablePeerAccess(c.device, 0);
+        cudaGetLastError();  // already enabled / unsupported: peer copies still work via the host
+      }
+      if (cudaMalloc(&x.h_pool, L * 2 * S * H * el) != cudaSuccess || dalloc(&x.c_pool, L * S * H) != cudaSuccess ||
+          dalloc(&x.tok, S) != cudaSuccess || dalloc(&x.dead, S) != cudaSuccess ||
+          dalloc(&x.ring_dev, E.ring_rows) != cudaSuccess || dalloc(&x.rows_flag_dev, 1) != cudaSuccess ||
+          cudaHostAlloc(reinterpret_cast<void**>(&x.ring_host), E.ring_rows * sizeof(RowDesc), cudaHostAllocDefault) !=
+              cudaSuccess ||
+          cudaHostAlloc(reinterpret_cast<void**>(&x.rows_seq_host), 256 * sizeof(unsigned int), cudaHostAllocDefault) !=
+              cudaSuccess ||
+          cudaStreamCreateWithFlags(&x.copy_stream, cudaStreamNonBlocking) != cudaSuccess ||
+          cudaEventCreateWithFlags(&x.copy_ev, cudaEventDisableTiming) != cudaSuccess)
+        return fail(BM_E_NOMEM);
+      if (cudaMemset(x.h_pool, 0, L * 2 * S * H * el) != cudaSuccess || cudaMemset(x.c_pool, 0, L * S * H * 4) != cudaSuccess ||
+          cudaMemset(x.tok, 0, S * 4) != cudaSuccess || cudaMemset(x.dead, 0, S * 4) != cudaSuccess ||
+          cudaMemset(x.rows_flag_dev, 0, 4) != cudaSuccess)
+        return fail(BM_E_CUDA);
+    }
+    if (c.devices > 1) {
+      cudaSetDevice(c.device);
+      for (int ci = 1; ci < c.devices; ++ci)
+        if (E.ctxs[ci].cuda_dev != c.device) {
+          cudaDeviceEnablePeerAccess(E.ctxs[ci].cuda_dev, 0);
+          cudaGetLastError();
+        }
+    }
+    // workers 1..W-1 (§8f N2): own stream, completion counter, launch chain, device scratch,
+    // allocated on the worker's context device
     for (int w = 1; w < c.workers; ++w) {
       WorkerState& ws = E.parked[w];
+      if (cudaSetDevice(E.ctxs[E.worker_ctx[w]].cuda_dev) != cudaSuccess) return fail(BM_E_CUDA);
       if (cudaStreamCreateWithFlags(&ws.stream, cudaStreamNonBlocking) != cudaSuccess ||
           cudaHostAlloc(reinterpret_cast<void**>(&ws.signal_host), kSignalSlots * sizeof(unsigned long long),
                         cudaHostAllocMapped) != cudaSuccess)
@@ -759,12 +911,11 @@ bm_status bm_create(const bm_config* cfg, bm_engine** out) {
           (c.precision == BM_PREC_BF16 &&
            dalloc(&ws.scratch, static_cast<size_t>(kPairScratchCTAs) * 128 * 256) != cudaSuccess))
         return fail(BM_E_NOMEM);
-      if (cudaMemsetAsync(ws.dep_flag, 0, 4, E.stream) != cudaSuccess ||
-          cudaMemsetAsync(ws.sig_ctas, 0, 4, E.stream) != cudaSuccess ||
-          cudaMemsetAsync(ws.done_ctas, 0, 4, E.stream) != cudaSuccess ||
-          cudaMemsetAsync(ws.amax, 0, 512 * 8, E.stream) != cudaSuccess)
+      if (cudaMemset(ws.dep_flag, 0, 4) != cudaSuccess || cudaMemset(ws.sig_ctas, 0, 4) != cudaSuccess ||
+          cudaMemset(ws.done_ctas, 0, 4) != cudaSuccess || cudaMemset(ws.amax, 0, 512 * 8) != cudaSuccess)
         return fail(BM_E_CUDA);
     }
+    cudaSetDevice(c.device);
     if (cudaStreamSynchronize(E.stream) != cudaSuccess) return fail(BM_E_CUDA);
   }
   *out = reinterpret_cast<bm_engine*>(e);
@@ -910,8 +1061,38 @@ bm_status bm_load_cell(bm_engine* h, const bm_cell_desc* d, const bm_weights* w,
     }
     cudaFree(tmp);
     cudaFree(tmpb);
+    // weight replica on every other device context (§8f N2): the packed bytes, peer-copied
+    for (size_t ci = 1; ci < e.ctxs.size(); ++ci) {
+      DevCtx& x = e.ctxs[ci];
+      CellWeights rep;
+      const int dd = x.cuda_dev, sd = e.cfg.device;
+      CK(cudaSetDevice(dd));
+      auto clone = [&](const void* src, size_t bytes, void** dst) -> cudaError_t {
+        *dst = nullptr;
+        if (src == nullptr) return cudaSuccess;
+        cudaError_t r = cudaMalloc(dst, bytes);
+        return r != cudaSuccess ? r : cudaMemcpyPeer(*dst, dd, src, sd, bytes);
+      };
+      for (int l = 0; l < L; ++l) {
+        void* wp = nullptr;
+        void* bp = nullptr;
+        CK(clone(c.W[l], rows * K * el, &wp));
+        CK(clone(c.bias[l], rows * 4, &bp));
+        rep.W.push_back(wp);
+        rep.bias.push_back(static_cast<float*>(bp));
+      }
+      void* b_out = nullptr;
+      CK(clone(c.E, static_cast<size_t>(d->vocab) * H * el, &rep.E));
+      CK(clone(c.W_out, static_cast<size_t>(d->vocab) * H * el, &rep.W_out));
+      CK(clone(c.b_out, static_cast<size_t>(d->vocab) * 4, &b_out));
+      rep.b_out = static_cast<float*>(b_out);
+      x.cells.resize(e.cells.size());
+      x.cells.push_back(rep);
+      CK(cudaSetDevice(sd));
+    }
   }
   e.cells.push_back(c);
+  for (size_t ci = 1; ci < e.ctxs.size(); ++ci) e.ctxs[ci].cells.resize(e.cells.size());
   *cell_id = static_cast<int>(e.cells.size()) - 1;
   return BM_OK;
 }

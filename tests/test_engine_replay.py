@@ -240,3 +240,47 @@ def test_replay_admits_due_arrivals_in_trace_order():
     rp = Replay([(4, 0)], max_slots=8).run(reqs)
     assert rp.tasks[0].tick == 0.0 and len(rp.tasks[0].rows) == 1
     assert sorted(t for _, t in rp.completions) == [1.0, 4.0]
+
+
+@settings(max_examples=150, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 100_000), n=st.integers(1, 20),
+       bmax=st.lists(st.integers(1, 6), min_size=5, max_size=5),
+       prio=st.permutations([0, 1, 2, 3, 4]), max_tasks=st.integers(1, 5),
+       k=st.integers(0, 3), slots=st.integers(4, 40), workers=st.integers(2, 4), devices=st.integers(2, 4),
+       kinds=st.sampled_from([[CHAIN], [SEQ2SEQ], [TREE], [CHAIN, SEQ2SEQ, TREE]]), eos=st.booleans())
+def test_multi_device_traces_bit_exact(seed, n, bmax, prio, max_tasks, k, slots, workers, devices, kinds, eos):
+    """§8f N2 across GPUs (L317, L337): W workers spread over D device contexts (worker w on
+    context w % D). Scheduling is Algorithm 1 as with one device -- the task log (worker by
+    worker), slots and completions equal the replay -- and the state rows moved between
+    contexts (an unpinned subgraph scheduled on another device, L337/L381; tree children
+    computed elsewhere) are exactly the replay's count."""
+    devices = min(devices, workers)
+    reqs = _random_reqs(seed, n, kinds, eos=eos)
+    need = max((len(q["left"]) if q["kind"] == TREE else 1) for q in reqs)
+    slots = max(slots, need)
+    kinds_c = [bm.CELL_LSTM, bm.CELL_LSTM, bm.CELL_LSTM_PROJ, bm.CELL_TREE_LEAF, bm.CELL_TREE_INTERNAL]
+    e, _ = _engine(list(zip(kinds_c, bmax, prio)), max_slots=slots, max_requests=64,
+                   max_tasks_to_submit=max_tasks, schedule_when_outstanding_leq=k, workers=workers,
+                   devices=devices)
+    _submit_all(e, reqs)
+    e.run()
+    rp = Replay(list(zip(bmax, prio)), max_slots=slots, max_tasks_to_submit=max_tasks,
+                schedule_when_outstanding_leq=k, workers=workers, devices=devices).run(reqs)
+    _compare(e, rp)
+    assert e.stats()["migrations"] == rp.migrations
+
+
+def test_multi_device_migrations_happen():
+    """A hand-checkable case: three 3-step chain requests arriving at ticks 0, 1, 2, bmax 1,
+    MaxTasksToSubmit 1, two workers on two device contexts. Worker 1 runs request 1's first two
+    steps; at tick 3 request 1 is unpinned and worker 0 (first in id order) takes its last step
+    -> one move; request 2 starts on worker 1 and continues on worker 0 -> a second move."""
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": float(i), "length": 3} for i in range(3)]
+    e, _ = _engine([(bm.CELL_LSTM, 1, 0)], max_slots=8, max_requests=8, workers=2, devices=2,
+                   max_tasks_to_submit=1)
+    _submit_all(e, reqs)
+    e.run()
+    rp = Replay([(1, 0)], max_slots=8, workers=2, devices=2, max_tasks_to_submit=1).run(reqs)
+    _compare(e, rp)
+    assert [(t.worker, [(r.rid, r.node) for r in t.rows]) for t in rp.tasks][5:7] == [(0, [(1, 2)]), (1, [(2, 0)])]
+    assert e.stats()["migrations"] == rp.migrations == 2

@@ -436,3 +436,75 @@ def test_weights_adopted_from_device_pointers():
     np.testing.assert_array_equal(out[0][1], out[1][1])
     hs, cs = cells.lstm_cell(w.W[0], w.b[0], w.E[rows[0, 0]], np.zeros(h), np.zeros(h))
     assert np.max(np.abs(out[1][0][0, 0] - hs)) <= 2e-4
+
+
+def test_two_devices_chain_and_trees_h1024():
+    """§8f N2 across GPUs, functional on one B200: two workers on two DEVICE CONTEXTS (each with
+    its own weight replica and state pool; on a multi-GPU box they are two GPUs). A subgraph
+    scheduled on the other context carries its state rows along (peer copies, L337). The task
+    log equals the replay worker for worker, the moves equal the replay's count (> 0), and every
+    request's result equals the oracle -- wrong or missing migrations would corrupt them."""
+    # sparse arrivals: a chain subgraph is pinned while a task of it is in flight (L381), so it
+    # only changes worker when it goes idle between tasks; at rate 0.3 that happens (4 moves)
+    trace = gen.chain_trace(48, 2048, seed=1003, rate=0.3)
+    e, cid, w = lstm_engine(1024, 1, 2048, bm.PREC_BF16, bmax=64, clock=bm.CLOCK_VIRTUAL, max_slots=256,
+                            max_requests=256, keep_results=1, max_tasks_to_submit=1, workers=2, devices=2)
+    for q in trace:
+        e.submit(bm.REQ_CHAIN, cid, 0, q.tokens, q.arrival)
+    e.run()
+    reqs = [{"kind": CHAIN, "cells": [0], "arrival": q.arrival, "length": q.length} for q in trace]
+    rp = Replay([(64, 0)], max_slots=256, max_tasks_to_submit=1, workers=2, devices=2).run(reqs)
+    _check_log(e, rp)
+    assert e.stats()["migrations"] == rp.migrations > 0
+    worst = 0.0
+    for i, q in enumerate(trace):
+        r = e.read_result(i, 1)
+        hs, cs = cells.chain_lstm(w, q.tokens)
+        worst = max(worst, np.max(np.abs(r["h"][0] - hs[0])), np.max(np.abs(r["c"][0] - cs[0])))
+    assert worst <= TOL[bm.PREC_BF16], worst
+    e.close()
+    # trees: leaves and internal levels spread over the two contexts
+    tt = gen.tree_trace(24, 1000, seed=8, rate=2.0)
+    e, (leaf, intern), tw = tree_engine(1024, 1000, bm.PREC_BF16, bmax=16, clock=bm.CLOCK_VIRTUAL, max_slots=2048,
+                                        max_requests=64, keep_results=1, max_tasks_to_submit=1, workers=2, devices=2)
+    for q in tt:
+        e.submit(bm.REQ_TREE, leaf, intern, q.tokens, q.arrival, left=q.left, right=q.right)
+    e.run()
+    rq = [{"kind": TREE, "cells": [0, 1], "arrival": q.arrival, "left": q.left, "right": q.right} for q in tt]
+    rp = Replay([(16, 0), (16, 1)], max_slots=2048, max_tasks_to_submit=1, workers=2, devices=2).run(rq)
+    _check_log(e, rp)
+    assert e.stats()["migrations"] == rp.migrations > 0
+    for i, q in enumerate(tt):
+        r = e.read_result(i, 1)
+        rh, rc, _ = cells.tree_lstm(tw, q.tokens, q.left, q.right)
+        assert np.max(np.abs(r["h"][0] - rh)) <= TOL[bm.PREC_BF16] and np.max(np.abs(r["c"][0] - rc)) <= TOL[bm.PREC_BF16]
+
+
+def test_two_devices_seq2seq_eos():
+    """Two device contexts with the Seq2Seq decoder: the feed token and the <eos> mark move with
+    the request's state rows (greedy feed-previous stays on the token the device emitted)."""
+    h, V, L = 64, 256, 4
+    trace = _s2s_trace(V, 12, 98)
+    kw = dict(bmax=(4, 4), clock=bm.CLOCK_VIRTUAL, max_slots=64, max_requests=64, keep_results=1,
+              max_decode_len=40, workers=2, devices=2, max_tasks_to_submit=1)
+    e, (ce, cd), (enc, dec) = seq2seq_engine(h, L, V, bm.PREC_BF16, **kw)
+    eos = 7
+    for toks, T, t in trace:
+        e.submit(bm.REQ_SEQ2SEQ, ce, cd, toks, t, decode_len=T, eos_id=eos)
+    e.run()
+    steps = []
+    for i, (toks, T, _) in enumerate(trace):
+        r = e.read_result(i, L, decode_len=T)
+        y = [int(v) for v in r["tokens"]]
+        m = y.index(-1) if -1 in y else T
+        steps.append(m - 1 if (m < T or y[T - 1] == eos) else None)
+        o = cells.seq2seq(enc, dec, toks, T, forced_tokens=y[:m], eos_id=eos)
+        for s in range(m):
+            assert o["logits"][s][y[s]] >= o["logits"][s].max() - 2 * TOL[bm.PREC_BF16]
+        for l in range(L):
+            assert np.max(np.abs(r["h"][l] - o["h"][l])) <= TOL[bm.PREC_BF16]
+    reqs = [{"kind": SEQ2SEQ, "cells": [0, 1], "arrival": t, "length": len(toks), "decode_len": T,
+             "eos_step": steps[i]} for i, (toks, T, t) in enumerate(trace)]
+    rp = Replay([(4, 0), (4, 1)], max_slots=64, workers=2, devices=2, max_tasks_to_submit=1).run(reqs)
+    _check_log(e, rp)
+    assert e.stats()["migrations"] == rp.migrations > 0
