@@ -11,8 +11,12 @@ makes one of them the headline instead.
 Protocol (L423 "adjust the average inter-arrival time", L489 p90 vs throughput):
   1. saturation estimate mu: a burst trace (every request arrives at t = 0);
   2. sustained load sweep, untimed: offered rate lambda on a grid of fractions of mu, each point
-     an open-loop Poisson trace of >= 100 k requests or >= 5 s; a point is SUSTAINED when the
-     achieved rate is within 2% of the offered one (no backlog growth); p50/p90/p99 per point;
+     an open-loop Poisson trace of >= 200 k requests or >= 5 s; a point is SUSTAINED when the
+     steady-state completion rate (completions between the arrival at 10% of the trace and the
+     last arrival, per second; steady_rate) is within 2% of the offered one AND the backlog
+     (arrived, not completed) at the last arrival is at most 1.3x the mid-window backlog (+64)
+     -- no backlog growth; the drain after the last arrival is reported, not charged;
+     p50/p90/p99 per point;
   3. lambda* = the highest sustained offered rate whose p90 is within the bound (12 ms, the
      paper's flat-region LSTM p90, L489; Seq2Seq: the knee, 2x the lowest-load p90), refined
      by bisection against the next (failing) grid point;
@@ -66,9 +70,10 @@ sys.path.insert(0, ROOT)
 from workloads import gen  # noqa: E402
 
 METRIC = "requests/sec at p90-latency bound"
-POINT_REQS = 100_000     # sweep point: >= 100 k requests ...
+POINT_REQS = 200_000     # sweep point: >= 200 k requests ...
 POINT_SECONDS = 5.0      # ... or >= 5 s of offered load, whichever is reached first
 SUSTAINED = 0.98         # achieved / offered of a sustained point
+BACKLOG_GROWTH = 1.3     # backlog at the last arrival / backlog at mid-window of a sustained point
 
 
 def parse():
@@ -446,15 +451,43 @@ class Ctx:
     pass
 
 
+def steady_rate(comp):
+    """Completion rate in the steady-state window: completions between the arrival of the
+    request at 10% of the trace and the LAST arrival, per second of that window. An open-loop
+    point whose system keeps up completes requests at the offered rate inside the window; an
+    overloaded one completes them at its capacity and its backlog grows. n / wall (first arrival
+    to last completion) also charges the drain of the last, longest requests (~p99 latency)
+    to the rate, which is no backlog. Returns (rate, backlog at mid-window, backlog at the end)."""
+    ta = np.sort(comp["t_arrival"])
+    td = comp["t_done"]
+    t0, t1 = ta[len(ta) // 10], ta[-1]
+    if t1 <= t0:
+        return float("nan"), 0, 0
+    tm = 0.5 * (t0 + t1)
+    rate = float(np.count_nonzero((td >= t0) & (td <= t1))) / (t1 - t0)
+    backlog = [int(np.searchsorted(ta, t, side="right") - np.count_nonzero(td <= t)) for t in (tm, t1)]
+    return rate, backlog[0], backlog[1]
+
+
 def measure_point(ctx, e, prep, n, lam):
-    """One open-loop Poisson point at offered rate lam (unit-rate trace rescaled)."""
+    """One open-loop Poisson point at offered rate lam (unit-rate trace rescaled). SUSTAINED =
+    the steady-state completion rate is within 2% of the offered rate (steady_rate)."""
     prep.set_time_scale(1.0 / lam)
     wall, comp = run_trace(e, prep, n, ctx.dry)
     lat = comp["t_done"] - comp["t_arrival"]
     p50, p90, p99 = (ctx.allmax(pct(lat, q)) for q in (50, 90, 99))
-    achieved = ctx.allmin(n / wall)
-    return {"offered": lam, "achieved": achieved, "n": n, "seconds": wall, "p50_ms": p50 * 1e3,
-            "p90_ms": p90 * 1e3, "p99_ms": p99 * 1e3, "sustained": bool(achieved >= SUSTAINED * lam)}
+    rate, b_mid, b_end = steady_rate(comp)
+    if ctx.dry:   # virtual ticks: the steady window is in ticks, not seconds
+        rate = float("nan")
+    achieved = ctx.allmin(rate) if rate == rate else ctx.allmin(n / wall)
+    # no backlog growth: the requests in the system at the last arrival are at most
+    # BACKLOG_GROWTH x those at mid-window (+ one task's worth of Poisson noise)
+    b_mid, b_end = ctx.allmax(b_mid), ctx.allmax(b_end)
+    steady = ctx.dry or b_end <= BACKLOG_GROWTH * b_mid + 64
+    return {"offered": lam, "achieved": achieved, "achieved_incl_drain": ctx.allmin(n / wall), "n": n,
+            "seconds": wall, "backlog_mid": int(b_mid), "backlog_end": int(b_end), "p50_ms": p50 * 1e3,
+            "p90_ms": p90 * 1e3, "p99_ms": p99 * 1e3,
+            "sustained": bool(achieved >= SUSTAINED * lam and steady)}
 
 
 def run_workload(ctx, a, wl, n_req, steps, warmup, headline):
@@ -533,8 +566,8 @@ def run_workload(ctx, a, wl, n_req, steps, warmup, headline):
         lam_star = lo
         curve.sort(key=lambda c: c["offered"])
         bounds = {"12ms": best_under(12.0), "knee": best_under(knee_ms), "knee_ms": knee_ms,
-                  "rule": f"highest offered rate with achieved >= {SUSTAINED:.0%} of offered and p90 within "
-                          "the bound; points of >= 100 k requests or >= 5 s"}
+                  "rule": f"highest offered rate with steady-state completion rate >= {SUSTAINED:.0%} of "
+                          "offered, backlog growth <= 1.3x, and p90 within the bound; points of >= 200 k requests or >= 5 s"}
     # ---- 4. timed steps at lambda*
     trace = make_trace(wl, n_req, 1.0, seed=ctx.shard.rank_seed(1000, rank))
     prep = e.prepare_requests(trace, cells)
@@ -568,7 +601,7 @@ def run_workload(ctx, a, wl, n_req, steps, warmup, headline):
             lats.append(comp["t_done"] - comp["t_arrival"])
             queue.append(comp["t_first"] - comp["t_arrival"])   # E5 (Fig. 9): queueing
             compute.append(comp["t_done"] - comp["t_first"])     # ... and computation time
-            achieved.append(n_req / wall)
+            achieved.append(steady_rate(comp)[0] if not ctx.dry else n_req / wall)
     ctx.barrier()
     st = e.stats()
     launch_log = None if ctx.dry else e.launch_log()

@@ -8,6 +8,8 @@
 #   bash tools/gpu.sh phases    [TAG]   BM_PHASE_DUMP phase timelines of LSTM steps (tools/phases.py)
 #   bash tools/gpu.sh stream            in-kernel L2/HBM -> shared streaming rates (tools/stream_bench.cu)
 #   bash tools/gpu.sh sanitize          compute-sanitizer memcheck / racecheck / synccheck over smoke()
+#   bash tools/gpu.sh sweep     [TAG]   kbench of one cell under each env plan in $PLANS (';'-separated,
+#                                       e.g. PLANS='BM_PAIR_XKB=1;BM_PAIR_WCPA=0 BM_PAIR_WS=4'), CELL, BS
 #
 # Outputs go to gpurun_out/ (merged back by gpurun); copy what is to be judged to profiles/.
 set -u
@@ -63,6 +65,17 @@ stream)
   for G in 1 2 4; do timeout 30 $S 7 16384 2 $L2 148 $G; done          # cp.async, G thread groups
   for G in 2 4; do timeout 30 $S 8 16384 2 $L2 148 $G; done            # TMA bulk, G issuing lanes
   for c in 16384 32768; do timeout 30 $S 3 $c 4 $L2 148 1; timeout 30 $S 4 $c 4 $L2 148 1; done  # tensor / gather4
+  ;;
+sweep)
+  IFS=';' read -ra PL <<< "${PLANS:-}"
+  for plan in "" "${PL[@]}"; do
+    echo "== plan: ${plan:-default}"
+    env $plan timeout 300 python tools/kbench.py --cell ${CELL:-lstm} --b ${BS:-192,256,384,512} --iters 200 \
+      > gpurun_out/sweep_tmp.log 2>&1
+    python tools/kb_table.py gpurun_out/sweep_tmp.log
+    grep -i "error\|Traceback" gpurun_out/sweep_tmp.log | head -3
+  done > gpurun_out/sweep_$TAG.log 2>&1
+  cat gpurun_out/sweep_$TAG.log
   ;;
 sanitize)
   for tool in memcheck racecheck synccheck; do
