@@ -47,6 +47,11 @@ constexpr int kThreads = kProducerThreads + 64;
 constexpr int kMaxCols = 256;           // batch columns per CTA (MMA N <= 256)
 constexpr int kWStageBytes = 128 * 128; // 128 weight rows x 128 B
 constexpr int kMaxS = 4;                // max split-K cluster size (K = 2h = 2048 -> 4 x 512)
+// split-K partial tiles in shared memory: [column][gate row] fp32 with a 132-float pitch, so the
+// epilogue's quad items (4 consecutive units = 16 floats of one column, 8 per column in a warp)
+// hit 8 distinct 16-B bank groups per wavefront (a 128-float pitch puts every column of a warp
+// on the same banks: 16-way conflicts)
+constexpr int kPPitch = 132;
 
 // Shared-memory plan (identical on host and device).
 // The weight stream and the activation gather use separate rings:
@@ -182,15 +187,19 @@ __global__ void __launch_bounds__(kThreads, 2)
     // the launch's own rows (independent of earlier launches) into the smem table: one 16-byte
     // parameter load per thread (parameter loads miss the constant cache and serialise per
     // address: each row is read once and then shared through shared memory)
+    // row load and dependency poll overlap: the row's global load is in flight while the chain
+    // flag is polled (one round trip less on the launch's critical path)
     if constexpr (!INL) rows_wait(p);
-    if (tid < ncols) rtab[tid] = row_at(p, rr, col0 + tid);
+    RowDesc r0{};
+    if (tid < ncols) r0 = row_at(p, rr, col0 + tid);
+    dep_wait(p);  // pool h/c and feed tokens are written by earlier launches
+    if (tid < ncols) rtab[tid] = r0;
     named_bar(1, kProducerThreads);
 #pragma unroll
     for (int i = 0; i < kItems; ++i) {
       const int row = min((tid + i * kProducerThreads) >> 3, ncols - 1);
       rd[i] = rtab[row];
     }
-    dep_wait(p);  // pool h/c and feed tokens are written by earlier launches
     // device span starts when the launch's dependent work may begin (after the PDL wait)
     if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
     if (tid == 0 && p.tl != nullptr) atomicMax(p.tl + 1, ~gtimer());
@@ -350,9 +359,10 @@ __global__ void __launch_bounds__(kThreads, 2)
       for (int c0 = cc0 + (warp >> 2) * 32; c0 < cc0 + PC && c0 < npad; c0 += 64) {
         float v[32];
         tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
+        const uint32_t Ps = smem_u32(P) + trow * 4;  // shared-space stores (not generic ST.E)
 #pragma unroll
         for (int i = 0; i < 32; ++i)
-          if (c0 + i < npad) P[(c0 - cc0 + i) * pitch + trow] = v[i];
+          if (c0 + i < npad) st_shared_f32(Ps + (c0 - cc0 + i) * pitch * 4, v[i]);
       }
     }
     tc_fence_before();
@@ -455,9 +465,10 @@ __global__ void __launch_bounds__(kThreads, 2)
         float v[32];
         tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
         if (trow < tile_rows) {
+          const uint32_t Ps = smem_u32(P) + prow * 4;  // shared-space stores (not generic ST.E)
 #pragma unroll
           for (int i = 0; i < 32; ++i)
-            if (c0 + i < npad) P[(c0 - cc0 + i) * pitch + prow] = v[i];
+            if (c0 + i < npad) st_shared_f32(Ps + (c0 - cc0 + i) * pitch * 4, v[i]);
         }
       }
     }
@@ -855,8 +866,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     // ================================================================ activation gather (A6)
     constexpr int kItems = 4;  // nhalf <= 128 rows x 8 chunks / 256 threads
     const int n_items = (nhalf * 8 + kProducerThreads - 1 - tid) / kProducerThreads;
+    // row load and dependency poll overlap (one round trip less on the critical path)
     if constexpr (!INL) rows_wait(p);
-    if (tid < ncols) rtab[tid] = row_at(p, rr, col0 + tid);
+    RowDesc r0{};
+    if (tid < ncols) r0 = row_at(p, rr, col0 + tid);
+    dep_wait(p);
+    if (tid < ncols) rtab[tid] = r0;
     named_bar(1, kProducerThreads);
     const __nv_bfloat16* src0[kItems];
     const __nv_bfloat16* src1[kItems];
@@ -864,7 +879,6 @@ __global__ void __launch_bounds__(kThreads, 1)
     RowDesc rd[kItems];
 #pragma unroll
     for (int i = 0; i < kItems; ++i) rd[i] = rtab[min(h0 + ((tid + i * kProducerThreads) >> 3), ncols - 1)];
-    dep_wait(p);
     if (tid == 0 && p.span != nullptr) atomicMin(p.span, gtimer());
     if (tid == 0) phase_mark(p, 8);
 #pragma unroll
@@ -909,14 +923,16 @@ __global__ void __launch_bounds__(kThreads, 1)
             cp_async_16(wdst + (tid + i * kProducerThreads) * 16, wsrc + (tid + i * kProducerThreads) * 16, 16);
         }
       }
-      if (st == 0) {
+      cp_async_arrive_noinc(full0 + 8 * s);
+      if (tid == 0 && st == 0) phase_mark(p, 10);
+      if (st == 0) {  // the epilogue's c rows, after stage 0's hand-off (off the first MMA's
+                      // path; covered by the next stage's arrive and the epilogue's wait_all):
+                      // -0.6 us per launch at b = 256..512 against issuing them with stage 0
         const int cper_ = (ncols + p.S - 1) / p.S;
         const int clo_ = ks * cper_;
         prefetch_c<EPI_LSTM>(p, rtab, clo_, max(0, min(ncols, clo_ + cper_) - clo_), tile * U,
                              smem_u32(base + p.cbuf_off), tid, kProducerThreads);
       }
-      cp_async_arrive_noinc(full0 + 8 * s);
-      if (tid == 0 && st == 0) phase_mark(p, 10);
     }
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
@@ -1025,14 +1041,15 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int S = p.S;
   const int cper = (ncols + S - 1) / S;
   float* P = reinterpret_cast<float*>(smem);
-  constexpr int pitch = 128;
-  if (warp < 8) {
+  constexpr int pitch = kPPitch;
+  if (warp < 8) {  // shared-space stores (a generic pointer into smem compiles to ST.E)
+    const uint32_t Ps = smem_u32(P) + trow * 4;
     for (int c0 = (warp >> 2) * 32; c0 < npad; c0 += 64) {
       float v[32];
       tmem_ld32(tmem + (static_cast<uint32_t>(32 * q) << 16) + c0, v);
 #pragma unroll
       for (int i = 0; i < 32; ++i)
-        if (c0 + i < npad) P[(c0 + i) * pitch + trow] = v[i];
+        if (c0 + i < npad) st_shared_f32(Ps + (c0 + i) * pitch * 4, v[i]);
     }
   }
   tc_fence_before();
@@ -1063,8 +1080,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (h < nit) {
           const uint32_t off = static_cast<uint32_t>(((c_lo + cl + h * ew) * pitch + j * G) * 4);
 #pragma unroll
-          for (int s = 0; s < kMaxS; ++s)
-            if (s < S) v[h][s] = ld_cluster_v4(peer[s] + off);
+          for (int s = 0; s < kMaxS; ++s)  // own partial through the local shared-memory path
+            if (s < S) v[h][s] = s == ks ? ld_shared_v4(smem_u32(P) + off) : ld_cluster_v4(peer[s] + off);
           r[h] = rtab[c_lo + cl + h * ew];
           cin[h] = cbuf[(cl + h * ew) * U + j];
         }
@@ -1218,7 +1235,7 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   if (stages < 2) return cudaSuccess;
   a.xring = stages * xstage;
   const int region = kWRing * a.wcb * 16 * 1024 + a.xring;
-  const int pbytes = cpb * 128 * 4;
+  const int pbytes = cpb * kPPitch * 4;
   a.cbuf_off = kTailBytes + (region > pbytes ? region : pbytes);
   const size_t need = 1024 + a.cbuf_off + ((((cpb + S - 1) / S) * a.U * 4 + 1023) & ~1023);
   if (need > static_cast<size_t>(smem)) return cudaSuccess;
