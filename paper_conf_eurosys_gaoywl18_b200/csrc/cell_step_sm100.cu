@@ -257,14 +257,14 @@ __global__ void __launch_bounds__(kThreads, 2)
             cp_async_16(wdst + i * 16, wsrc + i * 16, 16);
         }
       }
-      if (st == 0 && EPI != EPI_PROJ && p.pchunk == 0) {
-        const int cper_ = (ncols + p.S - 1) / p.S;
-        const int clo_ = static_cast<int>(rank) * cper_;
+      cp_async_arrive_noinc(full0 + 8 * s);
+      if (tid == 0 && st == 0) phase_mark(p, 10);
+      if (st == 0 && EPI != EPI_PROJ && p.pchunk == 0) {  // c rows after stage 0's hand-off
+        const int cper_ = (ncols + p.S - 1) / p.S;        // (covered by the next arrive and
+        const int clo_ = static_cast<int>(rank) * cper_;  // the epilogue's wait_all)
         prefetch_c<EPI>(p, rtab, clo_, max(0, min(ncols, clo_ + cper_) - clo_), blockIdx.y * U,
                         smem_u32(base + p.cbuf_off), tid, kProducerThreads);
       }
-      cp_async_arrive_noinc(full0 + 8 * s);
-      if (tid == 0 && st == 0) phase_mark(p, 10);
     }
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)

@@ -17,6 +17,8 @@ def main():
     ap.add_argument("--b", default="1,16,64,128,256,512")
     ap.add_argument("--iters", type=int, default=200)
     ap.add_argument("--fp32", action="store_true")
+    ap.add_argument("--vary-tokens", type=int, default=0,
+                    help="cycle through N row sets with fresh random tokens (embedding rows not L2-resident)")
     ap.add_argument("--out", default="")
     a = ap.parse_args()
     import torch
@@ -54,16 +56,20 @@ def main():
         else:
             toks = rng.integers(3, V, size=b)
             rows = np.stack([toks, np.zeros(b), slots, (np.arange(b) % 2) * bm.ROW_PARITY], 1)
-        for _ in range(5):
-            e.cell_step(cid, rows, sync=False)
+        row_sets = [rows]
+        if a.vary_tokens and a.cell != "internal":
+            row_sets = [np.stack([rng.integers(3, V, size=b), np.zeros(b), slots,
+                                  (np.arange(b) % 2) * bm.ROW_PARITY], 1) for _ in range(a.vary_tokens)]
+        for i in range(5):
+            e.cell_step(cid, row_sets[i % len(row_sets)], sync=False)
         torch.cuda.synchronize()
         e.reset_stats()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         import time as _t
         th0 = _t.perf_counter()
-        for _ in range(a.iters):
-            e.cell_step(cid, rows, sync=False)
+        for i in range(a.iters):
+            e.cell_step(cid, row_sets[i % len(row_sets)], sync=False)
         th1 = _t.perf_counter()
         ev1.record(stream)
         ev1.synchronize()
