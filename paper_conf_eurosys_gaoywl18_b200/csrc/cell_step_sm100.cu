@@ -353,6 +353,9 @@ __global__ void __launch_bounds__(kThreads, 2)
     // smaller footprint lets two CTAs share an SM, so all vocab tiles run in one wave)
     const int PC = p.pchunk > 0 ? min(p.pchunk, npad) : npad;
     const int v0 = blockIdx.y * 128;
+    float pbias[4];  // this lane's vocab rows of the tile (lane + 32 k)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) pbias[k] = p.bias[v0 + lane + 32 * k];
     for (int cc0 = 0; cc0 < npad; cc0 += PC) {
     if (cc0 > 0) __syncthreads();  // the previous chunk's column scans are done
     if (warp < 8) {
@@ -368,29 +371,76 @@ __global__ void __launch_bounds__(kThreads, 2)
     tc_fence_before();
     __syncthreads();
     if (tid == 0 && cc0 == 0) phase_mark(p, 3);
-    for (int c = cc0 + tid; c < min(ncols, cc0 + PC); c += kThreads) {
-      const RowDesc r = rtab[c];
-      float best = -INFINITY;
-      int besti = 0;
-      float* lg = nullptr;
-      const bool masked = (r.flags & ROW_EOS) && p.dead != nullptr && p.dead[r.slot];
-      if (p.logits != nullptr && !masked) {
-        const int step = (r.flags & ROW_EOS) ? row_step(r.b) : r.b;
-        lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + step) * p.V + v0;
+    const int chunk_cols = min(ncols, cc0 + PC) - cc0;
+    if (chunk_cols >= 96) {
+      // one thread per column: a serial scan of the tile's 128 vocab rows (strict '>' keeps
+      // the lowest index among equal maxima, S9); every thread has a column at this width
+      for (int c = cc0 + tid; c < min(ncols, cc0 + PC); c += kThreads) {
+        const RowDesc r = rtab[c];
+        float best = -INFINITY;
+        int besti = 0;
+        float* lg = nullptr;
+        const bool masked = (r.flags & ROW_EOS) && p.dead != nullptr && p.dead[r.slot];
+        if (p.logits != nullptr && !masked) {
+          const int step = (r.flags & ROW_EOS) ? row_step(r.b) : r.b;
+          lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + step) * p.V + v0;
+        }
+        for (int i = 0; i < 128; ++i) {
+          const float z = P[(c - cc0) * pitch + i] + p.bias[v0 + i];
+          if (lg != nullptr) lg[i] = z;
+          if (z > best) {
+            best = z;
+            besti = i;
+          }
+        }
+        uint32_t ob = __float_as_uint(best);
+        ob = (ob & 0x80000000u) ? ~ob : (ob | 0x80000000u);
+        const unsigned long long key =
+            (static_cast<unsigned long long>(ob) << 32) | (0xFFFFFFFFu - static_cast<uint32_t>(v0 + besti));
+        atomicMax(p.amax + col0 + c, key);
       }
-      for (int i = 0; i < 128; ++i) {
-        const float z = P[(c - cc0) * pitch + i] + p.bias[v0 + i];
-        if (lg != nullptr) lg[i] = z;
-        if (z > best) {  // strict: keeps the lowest index among equal maxima
-          best = z;
-          besti = i;
+    } else {
+      // narrow chunks: one warp per column: lane l scans vocab rows l, l + 32, l + 64, l + 96 (increasing, strict
+      // '>' keeps its lowest index), then a shuffle reduction takes the larger value and, on equal
+      // values, the lower index -- the same argmax (and lowest-index tie-break, S9) as a serial
+      // scan over the 128 rows, with 4 instead of 128 dependent steps per column
+      for (int c = cc0 + warp; c < min(ncols, cc0 + PC); c += kThreads / 32) {
+        const RowDesc r = rtab[c];
+        float* lg = nullptr;
+        const bool masked = (r.flags & ROW_EOS) && p.dead != nullptr && p.dead[r.slot];
+        if (p.logits != nullptr && !masked) {
+          const int step = (r.flags & ROW_EOS) ? row_step(r.b) : r.b;
+          lg = p.logits + (static_cast<size_t>(r.flags >> 8) * p.max_decode + step) * p.V + v0;
+        }
+        float best = -INFINITY;
+        int besti = 0;
+  #pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int i = lane + 32 * k;
+          const float z = P[(c - cc0) * pitch + i] + pbias[k];
+          if (lg != nullptr) lg[i] = z;
+          if (z > best) {  // strict: keeps the lowest index among equal maxima
+            best = z;
+            besti = i;
+          }
+        }
+  #pragma unroll
+        for (int off = 16; off > 0; off >>= 1) {
+          const float ob_ = __shfl_xor_sync(0xffffffffu, best, off);
+          const int oi = __shfl_xor_sync(0xffffffffu, besti, off);
+          if (ob_ > best || (ob_ == best && oi < besti)) {
+            best = ob_;
+            besti = oi;
+          }
+        }
+        if (lane == 0) {
+          uint32_t ob = __float_as_uint(best);
+          ob = (ob & 0x80000000u) ? ~ob : (ob | 0x80000000u);
+          const unsigned long long key =
+              (static_cast<unsigned long long>(ob) << 32) | (0xFFFFFFFFu - static_cast<uint32_t>(v0 + besti));
+          atomicMax(p.amax + col0 + c, key);
         }
       }
-      uint32_t ob = __float_as_uint(best);
-      ob = (ob & 0x80000000u) ? ~ob : (ob | 0x80000000u);
-      const unsigned long long key =
-          (static_cast<unsigned long long>(ob) << 32) | (0xFFFFFFFFu - static_cast<uint32_t>(v0 + besti));
-      atomicMax(p.amax + col0 + c, key);
     }
     }  // column chunks
     __threadfence();
