@@ -868,6 +868,12 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int n_chunks = (nk + kpc - 1) / kpc;
   constexpr int wblk_bytes = 128 * 128;
   const uint16_t pair_mask = static_cast<uint16_t>(3u << (crank & ~1u));
+  // WCPA with p.wcpa == 2: the weight K blocks of a stage (contiguous in the packed layout) move
+  // by ONE bulk copy of the otherwise idle TMA warp, issued as soon as the stage is free -- for
+  // the first ring's worth before the dependency wait -- while the producers' cp.async carry only
+  // the activation gather; the copy completes on the stage's full barrier (one more arrival +
+  // its bytes)
+  const bool wtma = WCPA && p.wcpa == 2;
 
   uint64_t* bars = reinterpret_cast<uint64_t*>(base);
   const uint32_t full0 = smem_u32(bars);                              // local producers
@@ -886,7 +892,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (tid == 0) phase_mark(p, 0);
   if (tid == 0) {
     for (int s = 0; s < pairk::kStagesMax; ++s) {
-      mbar_init(full0 + 8 * s, kProducerThreads);
+      mbar_init(full0 + 8 * s, kProducerThreads + (wtma ? 1 : 0));
       mbar_init(empty0 + 8 * s, 1);
       mbar_init(pfull0 + 8 * s, 1);
     }
@@ -964,7 +970,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             else cp_async_16(xs + dst_off[i], dummy, 0);  // zero fill (h0 = 0, padding)
           }
         }
-        if constexpr (WCPA) {  // this CTA's pre-swizzled 16 KB weight tile of K block k
+        if (WCPA && !wtma) {  // this CTA's pre-swizzled 16 KB weight tile of K block k
           const uint8_t* wsrc = static_cast<const uint8_t*>(p.W) +
                                 (static_cast<size_t>(tile) * ((p.K0 + p.K1) / kBK) + k / kBK) * wblk_bytes;
           const uint32_t wdst = smem_u32(x_st + s * x_stage_bytes + xkb * x_blk_bytes + j * wblk_bytes);
@@ -986,6 +992,21 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else if (warp == kTmaWarp) {
     // ================================================================ weight stream (A7)
+    if (wtma && lane == 0) {
+      const int kblocks = (p.K0 + p.K1) / kBK;
+      const uint8_t* wsrc =
+          static_cast<const uint8_t*>(p.W) + (static_cast<size_t>(tile) * kblocks + k_begin / kBK) * wblk_bytes;
+      const uint32_t bytes = static_cast<uint32_t>(xkb * wblk_bytes);
+      for (int st = 0; st < nst; ++st) {
+        const int s = st % kStages;
+        const int round = st / kStages;
+        if (round > 0) wait_bounded<false>(empty0 + 8 * s, (round - 1) & 1);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(full0 + 8 * s), "r"(bytes)
+                     : "memory");
+        bulk_load(smem_u32(x_st + s * x_stage_bytes + xkb * x_blk_bytes), wsrc + static_cast<size_t>(st) * bytes,
+                  bytes, full0 + 8 * s);
+      }
+    }
     if (!WCPA && lane == 0) {
       const int kblocks = (p.K0 + p.K1) / kBK;
       const uint8_t* wsrc =
@@ -1277,6 +1298,10 @@ cudaError_t launch_pair(StepArgs a, const RowDesc* rows_host, cudaStream_t st, b
   while (a.xkb > 1 && nk % a.xkb != 0) a.xkb >>= 1;
   int xstage = nhalf * 128 * a.xkb + (wcpa ? 16384 * a.xkb : 0);
   if (wcpa) a.wcb = 0;  // no TMA weight ring
+  // the stage's weight part by one bulk copy of the TMA warp (a.wcpa = 2; BM_PAIR_WTMA=0: by the
+  // producers' cp.async): -0.1..-0.2 us per launch at b = 192..512 (profiles/round2/wtma_r2.log)
+  static const int wtma = getenv("BM_PAIR_WTMA") ? atoi(getenv("BM_PAIR_WTMA")) : 1;
+  a.wcpa = wcpa ? (wtma ? 2 : 1) : 0;
   const int budget = smem - 1024 - kTailBytes - ((((cpb + S - 1) / S) * a.U * 4 + 1023) & ~1023);
   if (!wcpa && nk * 16 * 1024 + 2 * xstage <= budget && nk <= 8) a.wcb = nk / 2;  // whole slice resident
   if (!wcpa && env_wcb > 0) a.wcb = env_wcb;

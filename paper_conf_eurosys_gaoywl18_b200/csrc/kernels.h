@@ -85,7 +85,9 @@ struct StepArgs {
                               // are then no-ops); cleared by the request's first encoder step
   int* eos_host;              // host-mapped [max_requests]: decode step + 1 of the <eos>, or 0
   int pchunk;                 // split-K exchange chunk (columns), 0 = whole tile (BM_PCHUNK)
-  int wcpa;                   // LSTM single-CTA kernel: weights by cp.async in the stages
+  int wcpa;                   // LSTM single-CTA kernel: weights by cp.async in the stages;
+                              // CTA-pair kernel: 2 = the stage's weight part by one bulk copy
+                              // of the TMA warp (completion on the stage's full barrier)
   int small_plan;             // engine has >= 2 workers: LSTM launches use a <= 113 KB shared-
                               // memory plan (no CTA pairs) so two workers' CTAs share an SM
   int cbuf_off;               // set by the launcher: shared-memory offset (from the 1 KB-aligned
