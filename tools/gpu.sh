@@ -7,7 +7,7 @@
 #   bash tools/gpu.sh kbench    [TAG]   per-b device spans of every cell kernel (tools/kbench.py)
 #   bash tools/gpu.sh phases    [TAG]   BM_PHASE_DUMP phase timelines of LSTM steps (tools/phases.py)
 #   bash tools/gpu.sh stream            in-kernel L2/HBM -> shared streaming rates (tools/stream_bench.cu)
-#   bash tools/gpu.sh sanitize          compute-sanitizer memcheck / racecheck / synccheck over smoke()
+#   bash tools/gpu.sh sanitize          compute-sanitizer memcheck / synccheck / racecheck over the cell kernels
 #   bash tools/gpu.sh sweep     [TAG]   kbench of one cell under each env plan in $PLANS (';'-separated,
 #                                       e.g. PLANS='BM_PAIR_XKB=1;BM_PAIR_WCPA=0 BM_PAIR_WS=4'), CELL, BS
 #
@@ -78,10 +78,12 @@ sweep)
   cat gpurun_out/sweep_$TAG.log
   ;;
 sanitize)
-  for tool in memcheck racecheck synccheck; do
-    echo "== $tool"
-    timeout 1200 /usr/local/cuda/bin/compute-sanitizer --tool $tool --print-limit 20 \
-      python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | grep -E "ERROR SUMMARY|smoke ok|Error|error|hazard" | head -20
+  S=/usr/local/cuda/bin/compute-sanitizer
+  for tool in memcheck synccheck racecheck; do
+    echo "== $tool: tools/memcheck_small.py (single-CTA cells, Seq2Seq, tree)"
+    timeout 900 $S --tool $tool --print-limit 10 python tools/memcheck_small.py 2>&1 | grep -v "^\s*$" | tail -6
+    echo "== $tool: tools/pair_cmp.py (CTA-pair kernel, b = 129..512)"
+    timeout 900 $S --tool $tool --print-limit 10 python tools/pair_cmp.py /tmp/pc.npz 2>&1 | grep -v "^\s*$" | tail -6
   done
   ;;
 *)
